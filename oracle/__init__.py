@@ -1,0 +1,96 @@
+"""ORACLE -- TEST INFRASTRUCTURE ONLY (see sam_oracle.c for the citations and the contract).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference legs may
+import this package.  The product package (paper_conf_pldi_malekiyb16_b200) never imports it
+and it never imports the product package.
+
+scan(x, k, s, inclusive, phase=0, run=None) -> (y, run)
+    x      : 1-D numpy array, dtype int32 / int64 / float32 / float64
+    y      : uint32 / uint64 (reinterpret as int32/int64 for comparisons), float64 for fp32
+             data, np.longdouble for fp64 data
+    phase  : lane of x[0] (global index mod s)
+    run    : per-(pass, lane) running sums, k*s entries (accumulator dtype); pass the returned
+             `run` back in to continue a stream (chunk-outer nesting of the same loop).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "sam_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (plain C, IEEE semantics: no fast-math, no contraction)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-ffp-contract=off",
+                               "-fno-fast-math", "-o", tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        lib = ctypes.CDLL(build())
+        P = ctypes.c_void_p
+        for name in ("oracle_scan_u32", "oracle_scan_u64", "oracle_scan_f64acc", "oracle_scan_ldacc"):
+            fn = getattr(lib, name)
+            fn.argtypes = [P, ctypes.c_uint64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P]
+            fn.restype = ctypes.c_int
+        lib.oracle_sizeof_long_double.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+_ACC = {
+    np.dtype(np.int32): (np.uint32, "oracle_scan_u32"),
+    np.dtype(np.uint32): (np.uint32, "oracle_scan_u32"),
+    np.dtype(np.int64): (np.uint64, "oracle_scan_u64"),
+    np.dtype(np.uint64): (np.uint64, "oracle_scan_u64"),
+    np.dtype(np.float32): (np.float64, "oracle_scan_f64acc"),
+    np.dtype(np.float64): (np.longdouble, "oracle_scan_ldacc"),
+}
+
+
+def acc_dtype(dtype) -> np.dtype:
+    return np.dtype(_ACC[np.dtype(dtype)][0])
+
+
+def scan(x: np.ndarray, k: int, s: int = 1, inclusive: bool = True, phase: int = 0, run=None):
+    lib = _load()
+    x = np.ascontiguousarray(x)
+    acc, fname = _ACC[x.dtype]
+    if x.dtype.kind in "iu":
+        a = x.view(acc).copy() if x.dtype.itemsize == np.dtype(acc).itemsize else x.astype(acc)
+    else:
+        a = x.astype(acc)
+    if run is None:
+        run = np.zeros(k * s, dtype=acc)
+    else:
+        run = np.ascontiguousarray(run, dtype=acc)
+        assert run.size == k * s
+    rc = getattr(lib, fname)(a.ctypes.data, a.size, int(k), int(s), int(bool(inclusive)), int(phase),
+                             run.ctypes.data)
+    if rc != 0:
+        raise ValueError(f"oracle rejected arguments (rc={rc}): k={k} s={s} phase={phase}")
+    return a, run
+
+
+def scan_values(x: np.ndarray, k: int, s: int = 1, inclusive: bool = True) -> np.ndarray:
+    """Convenience: result reinterpreted in the input's signedness for ints."""
+    y, _ = scan(x, k, s, inclusive)
+    if x.dtype.kind in "iu":
+        return y.view(x.dtype)
+    return y
+
+
+def long_double_bytes() -> int:
+    return _load().oracle_sizeof_long_double()
