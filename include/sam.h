@@ -1,0 +1,141 @@
+/*
+ * sam.h -- C ABI of libsam.so: single-pass higher-order (order k) and tuple-based (tuple s)
+ * prefix sums on NVIDIA B200 (sm_100a).
+ *
+ * Method: Maleki, Yang & Burtscher, "Higher-Order and Tuple-Based Massively-Parallel Prefix
+ * Sums", PLDI'16.  Citations "P:<line>" are lines of the paper text.
+ *
+ * SEMANTICS (what every entry point computes)
+ *   Tuple s: element i of a stream belongs to lane m = (g + i) mod s, g being the
+ *   global index of the stream's first element (0 for sam_scan); the s lanes are independent.
+ *   Order 1, inclusive: y[i] = x[i] + y[previous element of the same lane].
+ *   Order 1, exclusive: y[i] = sum of the lane's elements strictly before i.
+ *   Order k: the order-1 operator applied k times; exclusive order k is the
+ *   order-1 exclusive operator applied k times, i.e. the inclusive result shifted by k lane
+ *   positions (reading R1).
+ *   Integers: two's-complement wraparound mod 2^w (reading R2) -- results are bit-exact and
+ *   independent of association order; SAM_I32/SAM_I64 may equally hold unsigned data.
+ *   Floats: IEEE arithmetic in the element type; association order follows the tile geometry
+ *   (reading R6); accuracy contract in DESIGN.md reading R7.
+ *
+ * MEMORY AND OWNERSHIP
+ *   `in`, `out`, payload buffers: device pointers (cudaMalloc / torch CUDA tensors) on the
+ *   current device, owned by the caller, aligned to the element size.  `in == out` (in-place)
+ *   is allowed; any other overlap is SAM_ERR_INVALID_ARG.  The library owns only a workspace
+ *   (tile status/state arrays, a few counters) cached per (device, stream), grown lazily and
+ *   kept for the life of the process (sam_release_workspaces frees it).  Calls on one stream
+ *   are ordered; calls on different streams use different workspaces and may run concurrently.
+ *   CUDA-graph capture is supported (the kernel resets its counters itself, no host state
+ *   changes between replays) provided the workspace was created before capture (make one
+ *   un-captured call, or call sam_prepare).
+ *
+ * ERRORS
+ *   Every entry point returns a sam_status.  Argument validation happens synchronously before
+ *   any CUDA call.  SAM_ERR_CUDA reports a launch/allocation failure; asynchronous device
+ *   faults surface at the caller's next synchronisation.  sam_last_error() returns a
+ *   thread-local description of the last failure on the calling thread.
+ */
+#ifndef SAM_H_
+#define SAM_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { SAM_I32 = 0, SAM_I64 = 1, SAM_F32 = 2, SAM_F64 = 3 } sam_dtype;
+
+typedef enum {
+    SAM_OK = 0,
+    SAM_ERR_INVALID_ARG = -1,  /* null pointer with n > 0, partial overlap, bad rank/nranks, misaligned */
+    SAM_ERR_UNSUPPORTED = -2,  /* order or tuple outside 1..8, unknown dtype */
+    SAM_ERR_CUDA = -3,         /* CUDA launch / runtime failure */
+    SAM_ERR_OOM = -4,          /* workspace allocation failed */
+    SAM_ERR_INTERNAL = -5
+} sam_status;
+
+/* `stream` is a cudaStream_t passed as an opaque pointer (NULL = legacy default stream). */
+typedef void* sam_stream_t;
+
+/*
+ * sam_scan -- single-GPU order-k, tuple-s, inclusive/exclusive scan of n scalars.
+ * One kernel launch, one read of `in` and one write of `out`, the
+ * inter-tile carries propagated by decoupled look-back.
+ *   dtype      element type of in/out (n elements each)
+ *   order      k, 1..8          tuple  s, 1..8          inclusive  nonzero = inclusive
+ *   n          number of scalars (not tuples); n = 0 is a no-op returning SAM_OK
+ * Asynchronous on `stream`.
+ */
+int sam_scan(sam_dtype dtype, int order, int tuple, int inclusive, const void* in, void* out,
+             uint64_t n, sam_stream_t stream);
+
+/*
+ * sam_scan_seeded -- sam_scan of a stream that continues an earlier one:
+ *   global_offset  g = global index of in[0] (lane of in[0] is g mod s)
+ *   seed           device pointer to order*tuple values of dtype, laid out [lane][order], the
+ *                  state (y_1..y_k) of each global lane at its last element BEFORE this stream
+ *                  (NULL = all zero, i.e. the stream starts the array)
+ *   final_state    optional device pointer (order*tuple values, [lane][order]) receiving the
+ *                  state of each lane at its last element of this stream (lanes with no
+ *                  element in the stream receive their seed), NULL = not wanted.
+ */
+int sam_scan_seeded(sam_dtype dtype, int order, int tuple, int inclusive, const void* in,
+                    void* out, uint64_t n, uint64_t global_offset, const void* seed,
+                    void* final_state, sam_stream_t stream);
+
+/* Make sure the workspace for (current device, stream) exists (optional; useful before graph
+ * capture).  `max_n` sizes it for streams of up to max_n elements. */
+int sam_prepare(sam_dtype dtype, int order, int tuple, uint64_t max_n, sam_stream_t stream);
+
+/*
+ * Host-buffer entry point (end-to-end path): `in_host` / `out_host` are host pointers
+ * (pinned memory recommended; pageable works but is slower).  The array is streamed through
+ * the GPU in chunks: H2D copy, seeded scan and D2H copy of consecutive chunks overlap on
+ * separate streams, the carry of chunk j seeding chunk j+1 on the device.  Synchronous:
+ * returns after out_host holds the result.  `stream` orders the work after prior work on it.
+ */
+int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const void* in_host,
+                  void* out_host, uint64_t n, sam_stream_t stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Sharded (multi-GPU) scan: contiguous shards in rank order.
+ *   1. sam_shard_state: read-only pass over the local shard -> payload (device memory,
+ *      sam_shard_payload_bytes bytes): [u64 n_local][u64 global_offset][order*tuple values,
+ *      [lane][order]], padded to a multiple of 16 B] = the zero-seeded state of each global lane at its last element of the
+ *      shard.
+ *   2. the caller all-gathers the payloads of all ranks (NCCL all_gather over NVLink), in
+ *      rank order, into one device buffer of nranks * payload_bytes bytes.
+ *   3. sam_shard_scan: folds the payloads of ranks < rank with the carry operator (lanes
+ *      with no element in a shard pass the state through) into this shard's seed and runs
+ *      the seeded single-pass scan (the binomial fix-up C(r+t-j, t-j) is fused into the
+ *      carry application).
+ * --------------------------------------------------------------------------------------- */
+size_t sam_shard_payload_bytes(sam_dtype dtype, int order, int tuple);
+
+int sam_shard_state(sam_dtype dtype, int order, int tuple, const void* in_local,
+                    uint64_t n_local, uint64_t global_offset, void* payload_dev,
+                    sam_stream_t stream);
+
+int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const void* in_local,
+                   void* out_local, uint64_t n_local, uint64_t global_offset,
+                   const void* all_payloads_dev, int rank, int nranks, sam_stream_t stream);
+
+/* Host-side fold of gathered payloads (host memory, same layout) into the seed of `rank`
+ * (host memory, order*tuple values [lane][order], lanes of global index mod s).  This is the
+ * same routine the device fold runs; exposed for CPU-side orchestration and tests. */
+int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* all_payloads_host,
+                           int rank, int nranks, void* seed_host);
+
+/* Diagnostics */
+const char* sam_last_error(void);
+const char* sam_version(void);
+int sam_release_workspaces(void);
+/* Kernel launches issued by this library on the calling process since load (for bench). */
+uint64_t sam_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SAM_H_ */

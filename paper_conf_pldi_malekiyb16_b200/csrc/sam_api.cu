@@ -1,0 +1,427 @@
+// sam_api.cu -- the C ABI of libsam.so (include/sam.h): argument validation, per-(device,
+// stream) workspaces, dispatch over (element type, order), the sharded entry points and the
+// host-buffer streaming pipeline.  Every arithmetic step of the scan runs in the CUDA kernels
+// of sam_kernel.cuh; this file only validates, allocates and launches.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <atomic>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+
+#include "sam.h"
+#include "sam_launch.cuh"
+
+namespace sam {
+template <typename T, int K> cudaError_t launch_scan_tk(const LaunchArgs&, uint64_t*);
+template <typename T> cudaError_t launch_fold(const void*, size_t, int, int, int, void*, cudaStream_t, uint64_t*);
+template <typename T> cudaError_t launch_payload_init(void*, uint64_t, uint64_t, int, int, const void*, int, void*,
+                                                      cudaStream_t, uint64_t*);
+}  // namespace sam
+
+namespace {
+
+thread_local std::string g_err;
+std::atomic<uint64_t> g_launches{0};
+constexpr const char* kVersion = "sam-b200 0.1 (sm_100a, single-pass decoupled look-back, order 1-8, tuple 1-8)";
+
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+int cuda_fail(cudaError_t e, const char* where) {
+    g_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return SAM_ERR_CUDA;
+}
+
+size_t elem_size(sam_dtype d) { return (d == SAM_I32 || d == SAM_F32) ? 4 : 8; }
+
+int validate_common(sam_dtype dtype, int order, int tuple) {
+    if ((int)dtype < 0 || (int)dtype > 3) return fail(SAM_ERR_UNSUPPORTED, "unknown dtype");
+    if (order < 1 || order > 8) return fail(SAM_ERR_UNSUPPORTED, "order must be in 1..8 (DESIGN.md R4)");
+    if (tuple < 1 || tuple > 8) return fail(SAM_ERR_UNSUPPORTED, "tuple must be in 1..8 (DESIGN.md R4)");
+    return SAM_OK;
+}
+
+int validate_buffers(sam_dtype dtype, const void* in, const void* out, uint64_t n, bool need_out) {
+    if (n == 0) return SAM_OK;
+    const size_t w = elem_size(dtype);
+    if (!in || (need_out && !out)) return fail(SAM_ERR_INVALID_ARG, "null buffer with n > 0");
+    if (((uintptr_t)in % w) != 0 || (need_out && ((uintptr_t)out % w) != 0))
+        return fail(SAM_ERR_INVALID_ARG, "buffers must be aligned to the element size");
+    if (n > (UINT64_MAX / 16)) return fail(SAM_ERR_INVALID_ARG, "n too large");
+    if (need_out && in != out) {
+        const uintptr_t a0 = (uintptr_t)in, a1 = a0 + n * w, b0 = (uintptr_t)out, b1 = b0 + n * w;
+        if (a0 < b1 && b0 < a1) return fail(SAM_ERR_INVALID_ARG, "in and out partially overlap (only in == out is allowed)");
+    }
+    return SAM_OK;
+}
+
+struct Workspace {
+    uint64_t* status = nullptr;
+    size_t status_cap = 0;  // tiles
+    void* aggv = nullptr;
+    void* inclv = nullptr;
+    size_t val_cap = 0;     // bytes each
+    unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32 + pad][epoch u64][seed 512 B]
+};
+
+std::mutex g_mu;
+std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+std::map<int, int> g_sms;
+
+int num_sms(int dev) {
+    auto it = g_sms.find(dev);
+    if (it != g_sms.end()) return it->second;
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    g_sms[dev] = n;
+    return n;
+}
+
+constexpr size_t CTR_BYTES = 32 + 8 * 8 * 8;
+
+// workspace of (current device, stream) with room for `tiles` tiles of `valbytes` values each
+int get_ws(cudaStream_t st, size_t tiles, size_t valbytes, Workspace** out, int* dev_out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    std::lock_guard<std::mutex> lk(g_mu);
+    Workspace*& ws = g_ws[std::make_pair(dev, st)];
+    if (!ws) ws = new Workspace();
+    if (!ws->ctr) {
+        e = cudaMalloc(&ws->ctr, CTR_BYTES);
+        if (e != cudaSuccess) return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e));
+        e = cudaMemsetAsync(ws->ctr, 0, CTR_BYTES, st);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+    }
+    if (tiles > ws->status_cap || valbytes > ws->val_cap) {
+        // grow (never shrink); old buffers may still be read by queued kernels on this stream
+        e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+        if (tiles > ws->status_cap) {
+            size_t cap = tiles + tiles / 4 + 64;
+            if (ws->status) cudaFree(ws->status);
+            ws->status = nullptr;
+            e = cudaMalloc(&ws->status, cap * sizeof(uint64_t));
+            if (e != cudaSuccess) { ws->status_cap = 0; return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e)); }
+            e = cudaMemsetAsync(ws->status, 0, cap * sizeof(uint64_t), st);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+            ws->status_cap = cap;
+        }
+        if (valbytes > ws->val_cap) {
+            size_t cap = valbytes + valbytes / 4 + 4096;
+            if (ws->aggv) cudaFree(ws->aggv);
+            if (ws->inclv) cudaFree(ws->inclv);
+            ws->aggv = ws->inclv = nullptr;
+            e = cudaMalloc(&ws->aggv, cap);
+            if (e == cudaSuccess) e = cudaMalloc(&ws->inclv, cap);
+            if (e != cudaSuccess) { ws->val_cap = 0; return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e)); }
+            ws->val_cap = cap;
+        }
+    }
+    *out = ws;
+    *dev_out = dev;
+    return SAM_OK;
+}
+
+template <typename T>
+cudaError_t dispatch_k(int k, const sam::LaunchArgs& a) {
+    uint64_t l = 0;
+    cudaError_t e = cudaErrorInvalidValue;
+    switch (k) {
+        case 1: e = sam::launch_scan_tk<T, 1>(a, &l); break;
+        case 2: e = sam::launch_scan_tk<T, 2>(a, &l); break;
+        case 3: e = sam::launch_scan_tk<T, 3>(a, &l); break;
+        case 4: e = sam::launch_scan_tk<T, 4>(a, &l); break;
+        case 5: e = sam::launch_scan_tk<T, 5>(a, &l); break;
+        case 6: e = sam::launch_scan_tk<T, 6>(a, &l); break;
+        case 7: e = sam::launch_scan_tk<T, 7>(a, &l); break;
+        case 8: e = sam::launch_scan_tk<T, 8>(a, &l); break;
+    }
+    g_launches += l;
+    return e;
+}
+
+// one scan-kernel launch for a stream of n elements at global offset g
+int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void* out, uint64_t n, uint64_t g,
+             const void* seed, void* final_state, int store_mode, cudaStream_t st) {
+    const size_t w = elem_size(dtype);
+    const sam::Geom geo = sam::make_geom(s, 15);
+    const uint64_t h = g % (uint64_t)s;
+    const size_t tiles = (size_t)((h + n + geo.T - 1) / geo.T);
+    Workspace* ws = nullptr;
+    int dev = 0;
+    int rc = get_ws(st, tiles, tiles * (size_t)s * (size_t)k * w, &ws, &dev);
+    if (rc != SAM_OK) return rc;
+    sam::LaunchArgs a;
+    a.in = in;
+    a.out = out;
+    a.n = n;
+    a.g = g;
+    a.seed = seed;
+    a.final_state = final_state;
+    a.s = s;
+    a.inclusive = inclusive ? 1 : 0;
+    a.store_mode = store_mode;
+    a.stream = st;
+    a.status = ws->status;
+    a.aggv = ws->aggv;
+    a.inclv = ws->inclv;
+    a.tile_ctr = (unsigned long long*)(ws->ctr);
+    a.done_ctr = (unsigned int*)(ws->ctr + 8);
+    a.epoch_ptr = (unsigned long long*)(ws->ctr + 16);
+    a.num_sms = num_sms(dev);
+    cudaError_t e;
+    switch (dtype) {
+        case SAM_I32: e = dispatch_k<uint32_t>(k, a); break;
+        case SAM_I64: e = dispatch_k<uint64_t>(k, a); break;
+        case SAM_F32: e = dispatch_k<float>(k, a); break;
+        default: e = dispatch_k<double>(k, a); break;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "scan kernel launch");
+    return SAM_OK;
+}
+
+int payload_init(sam_dtype dtype, void* payload, uint64_t n, uint64_t g, int k, int s, const void* seed,
+                 int write_header, void* final_state, cudaStream_t st) {
+    uint64_t l = 0;
+    cudaError_t e;
+    switch (dtype) {
+        case SAM_I32: e = sam::launch_payload_init<uint32_t>(payload, n, g, k, s, seed, write_header, final_state, st, &l); break;
+        case SAM_I64: e = sam::launch_payload_init<uint64_t>(payload, n, g, k, s, seed, write_header, final_state, st, &l); break;
+        case SAM_F32: e = sam::launch_payload_init<float>(payload, n, g, k, s, seed, write_header, final_state, st, &l); break;
+        default: e = sam::launch_payload_init<double>(payload, n, g, k, s, seed, write_header, final_state, st, &l); break;
+    }
+    g_launches += l;
+    return e == cudaSuccess ? SAM_OK : cuda_fail(e, "payload init launch");
+}
+
+int store_mode_for(const void* in, const void* out) {
+    return ((((uintptr_t)in) ^ ((uintptr_t)out)) & 15) == 0 ? sam::STORE_BULK : sam::STORE_STRIPED;
+}
+
+}  // namespace
+
+extern "C" {
+
+int sam_scan(sam_dtype dtype, int order, int tuple, int inclusive, const void* in, void* out, uint64_t n,
+             sam_stream_t stream) {
+    return sam_scan_seeded(dtype, order, tuple, inclusive, in, out, n, 0, nullptr, nullptr, stream);
+}
+
+int sam_scan_seeded(sam_dtype dtype, int order, int tuple, int inclusive, const void* in, void* out, uint64_t n,
+                    uint64_t global_offset, const void* seed, void* final_state, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    rc = validate_buffers(dtype, in, out, n, true);
+    if (rc) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (final_state) {
+        rc = payload_init(dtype, nullptr, n, global_offset, order, tuple, seed, 0, final_state, st);
+        if (rc) return rc;
+    }
+    if (n == 0) return SAM_OK;
+    return run_scan(dtype, order, tuple, inclusive, in, out, n, global_offset, seed, final_state,
+                    store_mode_for(in, out), st);
+}
+
+int sam_prepare(sam_dtype dtype, int order, int tuple, uint64_t max_n, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    const sam::Geom geo = sam::make_geom(tuple, 15);
+    const size_t tiles = (size_t)((max_n + tuple + geo.T - 1) / geo.T);
+    Workspace* ws = nullptr;
+    int dev = 0;
+    return get_ws((cudaStream_t)stream, tiles, tiles * (size_t)tuple * (size_t)order * elem_size(dtype), &ws, &dev);
+}
+
+size_t sam_shard_payload_bytes(sam_dtype dtype, int order, int tuple) {
+    if (validate_common(dtype, order, tuple)) return 0;
+    // header + values, rounded to 16 B so every rank's payload in the gathered buffer is aligned
+    return (16 + (size_t)order * (size_t)tuple * elem_size(dtype) + 15) / 16 * 16;
+}
+
+int sam_shard_state(sam_dtype dtype, int order, int tuple, const void* in_local, uint64_t n_local,
+                    uint64_t global_offset, void* payload_dev, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    rc = validate_buffers(dtype, in_local, nullptr, n_local, false);
+    if (rc) return rc;
+    if (!payload_dev) return fail(SAM_ERR_INVALID_ARG, "null payload");
+    cudaStream_t st = (cudaStream_t)stream;
+    void* fs = (unsigned char*)payload_dev + 16;
+    rc = payload_init(dtype, payload_dev, n_local, global_offset, order, tuple, nullptr, 1, fs, st);
+    if (rc || n_local == 0) return rc;
+    return run_scan(dtype, order, tuple, 1, in_local, nullptr, n_local, global_offset, nullptr, fs,
+                    sam::STORE_NONE, st);
+}
+
+int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const void* in_local, void* out_local,
+                   uint64_t n_local, uint64_t global_offset, const void* all_payloads_dev, int rank, int nranks,
+                   sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAM_ERR_INVALID_ARG, "rank/nranks out of range");
+    if (rank > 0 && !all_payloads_dev) return fail(SAM_ERR_INVALID_ARG, "null payloads");
+    rc = validate_buffers(dtype, in_local, out_local, n_local, true);
+    if (rc) return rc;
+    if (n_local == 0) return SAM_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const void* seed = nullptr;
+    if (rank > 0) {
+        Workspace* ws = nullptr;
+        int dev = 0;
+        rc = get_ws(st, 0, 0, &ws, &dev);
+        if (rc) return rc;
+        void* seedbuf = ws->ctr + 32;
+        const size_t pb = sam_shard_payload_bytes(dtype, order, tuple);
+        uint64_t l = 0;
+        cudaError_t e;
+        switch (dtype) {
+            case SAM_I32: e = sam::launch_fold<uint32_t>(all_payloads_dev, pb, rank, order, tuple, seedbuf, st, &l); break;
+            case SAM_I64: e = sam::launch_fold<uint64_t>(all_payloads_dev, pb, rank, order, tuple, seedbuf, st, &l); break;
+            case SAM_F32: e = sam::launch_fold<float>(all_payloads_dev, pb, rank, order, tuple, seedbuf, st, &l); break;
+            default: e = sam::launch_fold<double>(all_payloads_dev, pb, rank, order, tuple, seedbuf, st, &l); break;
+        }
+        g_launches += l;
+        if (e != cudaSuccess) return cuda_fail(e, "fold launch");
+        seed = seedbuf;
+    }
+    return run_scan(dtype, order, tuple, inclusive, in_local, out_local, n_local, global_offset, seed, nullptr,
+                    store_mode_for(in_local, out_local), st);
+}
+
+int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* all_payloads_host, int rank,
+                           int nranks, void* seed_host) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAM_ERR_INVALID_ARG, "rank/nranks out of range");
+    if (!seed_host || (rank > 0 && !all_payloads_host)) return fail(SAM_ERR_INVALID_ARG, "null buffer");
+    const size_t pb = sam_shard_payload_bytes(dtype, order, tuple);
+    const unsigned char* P = (const unsigned char*)all_payloads_host;
+    for (int m = 0; m < tuple; ++m) {
+        switch (dtype) {
+            case SAM_I32: sam::fold_payloads<uint32_t>(P, pb, rank, order, tuple, m, (uint32_t*)seed_host + m * order); break;
+            case SAM_I64: sam::fold_payloads<uint64_t>(P, pb, rank, order, tuple, m, (uint64_t*)seed_host + m * order); break;
+            case SAM_F32: sam::fold_payloads<float>(P, pb, rank, order, tuple, m, (float*)seed_host + m * order); break;
+            default: sam::fold_payloads<double>(P, pb, rank, order, tuple, m, (double*)seed_host + m * order); break;
+        }
+    }
+    return SAM_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// host-buffer streaming pipeline: H2D(j+1) | scan(j) | D2H(j-1) on three streams
+// ---------------------------------------------------------------------------------------------
+namespace {
+struct HostPipe {
+    static constexpr int NB = 3;
+    int dev = -1;
+    size_t chunk_bytes = 0;
+    unsigned char* buf[NB] = {nullptr, nullptr, nullptr};
+    unsigned char* state = nullptr;  // 2 x 512 B
+    cudaStream_t s_h2d = nullptr, s_cmp = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev_h2d[NB], ev_cmp[NB], ev_d2h[NB], ev_start;
+};
+std::mutex g_pipe_mu;
+std::map<int, HostPipe*> g_pipes;
+constexpr size_t kChunkBytes = size_t(128) << 20;
+
+int get_pipe(HostPipe** out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    HostPipe*& P = g_pipes[dev];
+    if (!P) {
+        P = new HostPipe();
+        P->dev = dev;
+        P->chunk_bytes = kChunkBytes;
+        for (int i = 0; i < HostPipe::NB; ++i) {
+            e = cudaMalloc(&P->buf[i], P->chunk_bytes);
+            if (e != cudaSuccess) return fail(SAM_ERR_OOM, "host pipeline buffers");
+            cudaEventCreateWithFlags(&P->ev_h2d[i], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&P->ev_cmp[i], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&P->ev_d2h[i], cudaEventDisableTiming);
+        }
+        e = cudaMalloc(&P->state, 1024);
+        if (e != cudaSuccess) return fail(SAM_ERR_OOM, "host pipeline state");
+        cudaEventCreateWithFlags(&P->ev_start, cudaEventDisableTiming);
+        cudaStreamCreateWithFlags(&P->s_h2d, cudaStreamNonBlocking);
+        cudaStreamCreateWithFlags(&P->s_cmp, cudaStreamNonBlocking);
+        cudaStreamCreateWithFlags(&P->s_d2h, cudaStreamNonBlocking);
+    }
+    *out = P;
+    return SAM_OK;
+}
+}  // namespace
+
+int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const void* in_host, void* out_host,
+                  uint64_t n, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (n == 0) return SAM_OK;
+    if (!in_host || !out_host) return fail(SAM_ERR_INVALID_ARG, "null buffer with n > 0");
+    std::lock_guard<std::mutex> lk(g_pipe_mu);
+    HostPipe* P = nullptr;
+    rc = get_pipe(&P);
+    if (rc) return rc;
+    const size_t w = elem_size(dtype);
+    const uint64_t C = P->chunk_bytes / w;
+    const uint64_t nchunks = (n + C - 1) / C;
+    cudaStream_t user = (cudaStream_t)stream;
+    cudaEventRecord(P->ev_start, user);
+    cudaStreamWaitEvent(P->s_h2d, P->ev_start, 0);
+    cudaStreamWaitEvent(P->s_cmp, P->ev_start, 0);
+    cudaStreamWaitEvent(P->s_d2h, P->ev_start, 0);
+    const size_t sb = (size_t)order * tuple * w;
+    for (uint64_t j = 0; j < nchunks; ++j) {
+        const int b = (int)(j % HostPipe::NB);
+        const uint64_t off = j * C;
+        const uint64_t cn = (n - off < C) ? n - off : C;
+        if (j >= (uint64_t)HostPipe::NB) cudaStreamWaitEvent(P->s_h2d, P->ev_d2h[b], 0);
+        cudaError_t e = cudaMemcpyAsync(P->buf[b], (const unsigned char*)in_host + off * w, cn * w,
+                                        cudaMemcpyHostToDevice, P->s_h2d);
+        if (e != cudaSuccess) return cuda_fail(e, "H2D");
+        cudaEventRecord(P->ev_h2d[b], P->s_h2d);
+        cudaStreamWaitEvent(P->s_cmp, P->ev_h2d[b], 0);
+        const void* seed = j ? (const void*)(P->state + ((j - 1) & 1) * 512) : nullptr;
+        void* fin = (j + 1 < nchunks) ? (void*)(P->state + (j & 1) * 512) : nullptr;
+        (void)sb;
+        rc = sam_scan_seeded(dtype, order, tuple, inclusive, P->buf[b], P->buf[b], cn, off, seed, fin, P->s_cmp);
+        if (rc) return rc;
+        cudaEventRecord(P->ev_cmp[b], P->s_cmp);
+        cudaStreamWaitEvent(P->s_d2h, P->ev_cmp[b], 0);
+        e = cudaMemcpyAsync((unsigned char*)out_host + off * w, P->buf[b], cn * w, cudaMemcpyDeviceToHost, P->s_d2h);
+        if (e != cudaSuccess) return cuda_fail(e, "D2H");
+        cudaEventRecord(P->ev_d2h[b], P->s_d2h);
+    }
+    cudaError_t e = cudaStreamSynchronize(P->s_d2h);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(P->s_cmp);
+    if (e != cudaSuccess) return cuda_fail(e, "host pipeline");
+    return SAM_OK;
+}
+
+const char* sam_last_error(void) { return g_err.c_str(); }
+const char* sam_version(void) { return kVersion; }
+uint64_t sam_launch_count(void) { return g_launches.load(); }
+
+int sam_release_workspaces(void) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    cudaDeviceSynchronize();
+    for (auto& kv : g_ws) {
+        Workspace* ws = kv.second;
+        if (ws->status) cudaFree(ws->status);
+        if (ws->aggv) cudaFree(ws->aggv);
+        if (ws->inclv) cudaFree(ws->inclv);
+        if (ws->ctr) cudaFree(ws->ctr);
+        delete ws;
+    }
+    g_ws.clear();
+    return SAM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,3 @@
+// Explicit instantiation of the scan kernel and launchers for element type uint32_t, orders 1..8.
+#include "sam_launch.cuh"
+SAM_INSTANTIATE(uint32_t)

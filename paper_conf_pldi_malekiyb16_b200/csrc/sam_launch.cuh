@@ -1,0 +1,177 @@
+// sam_launch.cuh -- host-side launch of the scan kernel for one (element type, order).
+// Instantiated per element type in sam_inst_*.cu; called by the C ABI in sam_api.cu.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "sam_algebra.h"
+#include "sam_kernel.cuh"
+
+namespace sam {
+
+// Tile geometry for tuple size s: a warp holds G lanes (G = largest power of two
+// dividing s) with Pw = 32/G threads per lane; sp = s/G lane groups; c warps per lane group.
+struct Geom {
+    int s, G, logG, sp, c, logc, Pw, W, Wn, Uw, U, T;
+};
+
+inline int ilog2(int x) {
+    int r = 0;
+    while ((1 << r) < x) ++r;
+    return r;
+}
+
+inline Geom make_geom(int s, int items) {
+    Geom g;
+    g.s = s;
+    g.G = s & -s;
+    g.logG = ilog2(g.G);
+    g.sp = s / g.G;
+    int c = 8 / g.sp;
+    if (c < 1) c = 1;
+    while (c & (c - 1)) c &= c - 1;  // power of two
+    g.c = c;
+    g.logc = ilog2(c);
+    g.W = g.sp * g.c;
+    g.Pw = 32 / g.G;
+    g.Uw = g.Pw * items;
+    g.U = g.c * g.Uw;
+    g.T = g.s * g.U;
+    g.Wn = 32 / s;
+    return g;
+}
+
+struct LaunchArgs {
+    const void* in;
+    void* out;
+    uint64_t n;
+    uint64_t g;            // global index of in[0]
+    const void* seed;      // [s][k] or null
+    void* final_state;     // [s][k] or null
+    int s;
+    int inclusive;
+    int store_mode;
+    cudaStream_t stream;
+    // workspace
+    uint64_t* status;
+    void* aggv;
+    void* inclv;
+    unsigned long long* tile_ctr;
+    unsigned int* done_ctr;
+    unsigned long long* epoch_ptr;
+    int num_sms;
+};
+
+template <typename T>
+inline int items_of() { return Cfg<T>::ITEMS; }
+
+template <typename T, int K>
+struct KernelInfo {
+    int max_blocks_per_sm = 0;
+    bool ready = false;
+    std::mutex mu;
+};
+
+template <typename T, int K>
+cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
+    using S = Smem<T, K>;
+    static KernelInfo<T, K> info;
+    {
+        std::lock_guard<std::mutex> lk(info.mu);
+        if (!info.ready) {
+            cudaError_t e = cudaFuncSetAttribute(sam_scan_kernel<T, K>,
+                                                 cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES);
+            if (e != cudaSuccess) return e;
+            int nb = 0;
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K>, MAX_THREADS, S::BYTES);
+            if (e != cudaSuccess) return e;
+            info.max_blocks_per_sm = nb > 0 ? nb : 1;
+            info.ready = true;
+        }
+    }
+    const Geom geo = make_geom(a.s, Cfg<T>::ITEMS);
+    Params<T, K> p;
+    memset(&p, 0, sizeof(p));
+    p.in = (const T*)a.in;
+    p.out = (T*)a.out;
+    p.n = a.n;
+    p.h = a.g % (uint64_t)a.s;
+    p.num_tiles = (p.h + a.n + geo.T - 1) / geo.T;
+    p.delta = (uint32_t)(((uintptr_t)a.in - p.h * sizeof(T)) & 15);
+    p.s = geo.s; p.G = geo.G; p.logG = geo.logG; p.sp = geo.sp; p.c = geo.c; p.logc = geo.logc;
+    p.Pw = geo.Pw; p.W = geo.W; p.Wn = geo.Wn; p.U = geo.U; p.T_ = geo.T; p.Uw = geo.Uw;
+    p.inclusive = a.inclusive;
+    p.store_mode = a.store_mode;
+    p.seed = (const T*)a.seed;
+    p.final_state = (T*)a.final_state;
+    for (int m = 0; m < MAXS; ++m) {
+        p.last_e[m] = -1;
+        if (m < a.s && a.n > 0) {
+            const int64_t eend = (int64_t)(p.h + a.n - 1);
+            const int64_t le = eend - ((eend - m) % a.s + a.s) % a.s;
+            if (le >= (int64_t)p.h && le >= 0) p.last_e[m] = le;
+        }
+    }
+    p.status = a.status;
+    p.aggv = (T*)a.aggv;
+    p.inclv = (T*)a.inclv;
+    p.tile_ctr = a.tile_ctr;
+    p.done_ctr = a.done_ctr;
+    p.epoch_ptr = a.epoch_ptr;
+    mcol<T>(Cfg<T>::ITEMS, K, p.bc);
+    mcol<T>(geo.Uw, K, p.bw);
+    mcol<T>(geo.U, K, p.bu);
+    mcol<T>((int64_t)geo.Wn * geo.U, K, p.bwin);
+    for (int v = 0; v < 32; ++v) {
+        T b[K];
+        mcol<T>((int64_t)v * Cfg<T>::ITEMS, K, b);
+        for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
+    }
+    for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
+    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
+
+    uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
+    if (grid > p.num_tiles) grid = p.num_tiles;
+    if (grid < 1) grid = 1;
+    sam_scan_kernel<T, K><<<(unsigned)grid, geo.W * 32, S::BYTES, a.stream>>>(p);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_fold(const void* payloads, size_t payload_bytes, int rank, int k, int s, void* seed,
+                        cudaStream_t st, uint64_t* launches) {
+    sam_fold_kernel<T><<<1, 32, 0, st>>>((const unsigned char*)payloads, payload_bytes, rank, k, s, (T*)seed);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_payload_init(void* payload, uint64_t n, uint64_t g, int k, int s, const void* seed,
+                                int write_header, void* final_state, cudaStream_t st, uint64_t* launches) {
+    sam_payload_init_kernel<T><<<1, 64, 0, st>>>((unsigned char*)payload, n, g, k, s, (const T*)seed,
+                                                 write_header, (T*)final_state);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+}  // namespace sam
+
+#define SAM_INSTANTIATE(T)                                                                             \
+    namespace sam {                                                                                    \
+    template cudaError_t launch_scan_tk<T, 1>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 2>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 3>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 4>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 5>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 6>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 7>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_scan_tk<T, 8>(const LaunchArgs&, uint64_t*);                           \
+    template cudaError_t launch_fold<T>(const void*, size_t, int, int, int, void*, cudaStream_t,       \
+                                        uint64_t*);                                                    \
+    template cudaError_t launch_payload_init<T>(void*, uint64_t, uint64_t, int, int, const void*, int, \
+                                                void*, cudaStream_t, uint64_t*);                       \
+    }

@@ -1,0 +1,96 @@
+"""Sharded (multi-GPU) scan over contiguous shards, SURVEY §8(e).
+
+One process per GPU.  Rank r holds elements [g_r, g_r + n_r) of the global array (rank order).
+
+    1. sam_shard_state   read-only pass over the local shard -> payload
+                         [u64 n_r][u64 g_r][k*s values] = zero-seeded state of each global lane
+                         at its last element in the shard (<= 16 + 512 bytes)
+    2. all_gather        NCCL all_gather_into_tensor of the payloads over NVLink / NVSwitch
+                         (the one exchange step of the path)
+    3. sam_shard_scan    fold of the payloads of ranks < r with the carry operator
+                         (M(L) s + v) into this shard's seed, then the seeded
+                         single-pass scan (binomial fix-up fused into the carry application)
+
+torch.distributed is plumbing only; every arithmetic step runs in libsam.so kernels.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+import torch.distributed as dist
+
+from . import (SamError, _stream_ptr, dtype_code, sam_shard_payload_bytes, sam_shard_scan, sam_shard_state)
+
+
+def shard_offsets(n_local: int, group=None, device=None) -> tuple[int, int]:
+    """(global offset of this rank's shard, global n) from an all-gather of the shard lengths."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    t = torch.tensor([n_local], dtype=torch.int64, device=device)
+    allv = torch.empty(world, dtype=torch.int64, device=device)
+    dist.all_gather_into_tensor(allv, t, group=group)
+    lens = allv.tolist()
+    return int(sum(lens[:rank])), int(sum(lens))
+
+
+def exchange_payloads(payload: torch.Tensor, group=None) -> torch.Tensor:
+    """All-gather the per-rank payloads (uint8) in rank order (NCCL over NVLink on GPUs)."""
+    world = dist.get_world_size(group)
+    gathered = torch.empty(world * payload.numel(), dtype=torch.uint8, device=payload.device)
+    dist.all_gather_into_tensor(gathered, payload, group=group)
+    return gathered
+
+
+def scan_sharded(x_local: torch.Tensor, order: int = 1, tuple: int = 1, inclusive: bool = True,
+                 group=None, global_offset: int | None = None, out: torch.Tensor | None = None,
+                 stream=None) -> torch.Tensor:
+    """Scan of the global array whose contiguous shard `x_local` this rank holds."""
+    if not x_local.is_cuda or x_local.dim() != 1 or not x_local.is_contiguous():
+        raise SamError(-1, "x_local must be a 1-D contiguous CUDA tensor")
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    if global_offset is None:
+        global_offset, _ = shard_offsets(x_local.numel(), group, device=x_local.device)
+    if out is None:
+        out = torch.empty_like(x_local)
+    dc = dtype_code(x_local.dtype)
+    st = _stream_ptr(stream)
+    n = x_local.numel()
+    if world == 1:
+        sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x_local.data_ptr()),
+                       ctypes.c_void_p(out.data_ptr()), n, global_offset, None, 0, 1, st)
+        return out
+    pb = sam_shard_payload_bytes(dc, order, tuple)
+    payload = torch.empty(pb, dtype=torch.uint8, device=x_local.device)
+    sam_shard_state(dc, order, tuple, ctypes.c_void_p(x_local.data_ptr()), n, global_offset,
+                    ctypes.c_void_p(payload.data_ptr()), st)
+    gathered = exchange_payloads(payload, group)
+    sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x_local.data_ptr()),
+                   ctypes.c_void_p(out.data_ptr()), n, global_offset, ctypes.c_void_p(gathered.data_ptr()),
+                   rank, world, st)
+    return out
+
+
+def scan_virtual_shards(x: torch.Tensor, bounds: list[int], order: int = 1, tuple: int = 1,
+                        inclusive: bool = True) -> torch.Tensor:
+    """Run the sharded schedule on ONE GPU over virtual shards x[bounds[i]:bounds[i+1]]
+    (state pass per shard, payload concatenation in place of the all-gather, seeded scans).
+    Exercises every multi-GPU code path except the NCCL transport."""
+    dc = dtype_code(x.dtype)
+    pb = sam_shard_payload_bytes(dc, order, tuple)
+    p = len(bounds) - 1
+    gathered = torch.empty(p * pb, dtype=torch.uint8, device=x.device)
+    out = torch.empty_like(x)
+    st = _stream_ptr()
+    w = x.element_size()
+    for r in range(p):
+        lo, hi = bounds[r], bounds[r + 1]
+        sam_shard_state(dc, order, tuple, ctypes.c_void_p(x.data_ptr() + lo * w), hi - lo, lo,
+                        ctypes.c_void_p(gathered.data_ptr() + r * pb), st)
+    for r in range(p):
+        lo, hi = bounds[r], bounds[r + 1]
+        sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x.data_ptr() + lo * w),
+                       ctypes.c_void_p(out.data_ptr() + lo * w), hi - lo, lo,
+                       ctypes.c_void_p(gathered.data_ptr()), r, p, st)
+    return out
