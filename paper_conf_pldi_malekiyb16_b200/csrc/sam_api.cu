@@ -61,12 +61,9 @@ int validate_buffers(sam_dtype dtype, const void* in, const void* out, uint64_t 
 }
 
 struct Workspace {
-    uint64_t* status = nullptr;
-    size_t status_cap = 0;  // tiles
-    void* aggv = nullptr;
-    void* inclv = nullptr;
-    size_t val_cap = 0;     // bytes each
-    unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32 + pad][epoch u64][seed 512 B]
+    unsigned long long* carry = nullptr;  // tagged carry words of every tile
+    size_t carry_cap = 0;                 // bytes
+    unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32][epoch u32][pad 16][seed 512 B]
 };
 
 std::mutex g_mu;
@@ -84,8 +81,8 @@ int num_sms(int dev) {
 
 constexpr size_t CTR_BYTES = 32 + 8 * 8 * 8;
 
-// workspace of (current device, stream) with room for `tiles` tiles of `valbytes` values each
-int get_ws(cudaStream_t st, size_t tiles, size_t valbytes, Workspace** out, int* dev_out) {
+// workspace of (current device, stream) with room for `carry_bytes` of tagged carry words
+int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
@@ -98,34 +95,38 @@ int get_ws(cudaStream_t st, size_t tiles, size_t valbytes, Workspace** out, int*
         e = cudaMemsetAsync(ws->ctr, 0, CTR_BYTES, st);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
     }
-    if (tiles > ws->status_cap || valbytes > ws->val_cap) {
-        // grow (never shrink); old buffers may still be read by queued kernels on this stream
+    if (carry_bytes > ws->carry_cap) {
+        // grow (never shrink); the old buffer may still be read by queued kernels on this stream
         e = cudaStreamSynchronize(st);
         if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
-        if (tiles > ws->status_cap) {
-            size_t cap = tiles + tiles / 4 + 64;
-            if (ws->status) cudaFree(ws->status);
-            ws->status = nullptr;
-            e = cudaMalloc(&ws->status, cap * sizeof(uint64_t));
-            if (e != cudaSuccess) { ws->status_cap = 0; return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e)); }
-            e = cudaMemsetAsync(ws->status, 0, cap * sizeof(uint64_t), st);
-            if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
-            ws->status_cap = cap;
-        }
-        if (valbytes > ws->val_cap) {
-            size_t cap = valbytes + valbytes / 4 + 4096;
-            if (ws->aggv) cudaFree(ws->aggv);
-            if (ws->inclv) cudaFree(ws->inclv);
-            ws->aggv = ws->inclv = nullptr;
-            e = cudaMalloc(&ws->aggv, cap);
-            if (e == cudaSuccess) e = cudaMalloc(&ws->inclv, cap);
-            if (e != cudaSuccess) { ws->val_cap = 0; return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e)); }
-            ws->val_cap = cap;
-        }
+        const size_t cap = carry_bytes + carry_bytes / 4 + 4096;
+        if (ws->carry) cudaFree(ws->carry);
+        ws->carry = nullptr;
+        ws->carry_cap = 0;
+        e = cudaMalloc(&ws->carry, cap);
+        if (e != cudaSuccess) return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e));
+        // zero words carry tag 0, which no launch uses
+        e = cudaMemsetAsync(ws->carry, 0, cap, st);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+        ws->carry_cap = cap;
     }
     *out = ws;
     *dev_out = dev;
     return SAM_OK;
+}
+
+int items_of(sam_dtype d) {
+    switch (d) {
+        case SAM_I32: return sam::Cfg<uint32_t>::ITEMS;
+        case SAM_I64: return sam::Cfg<uint64_t>::ITEMS;
+        case SAM_F32: return sam::Cfg<float>::ITEMS;
+        default: return sam::Cfg<double>::ITEMS;
+    }
+}
+
+// bytes of tagged carry words for `tiles` tiles: per (lane, order) 2 values x (1 or 2) words
+size_t carry_bytes(sam_dtype d, int k, int s, size_t tiles) {
+    return tiles * (size_t)s * (size_t)k * 2 * (elem_size(d) / 4) * 8;
 }
 
 template <typename T>
@@ -149,13 +150,12 @@ cudaError_t dispatch_k(int k, const sam::LaunchArgs& a) {
 // one scan-kernel launch for a stream of n elements at global offset g
 int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void* out, uint64_t n, uint64_t g,
              const void* seed, void* final_state, int store_mode, cudaStream_t st) {
-    const size_t w = elem_size(dtype);
-    const sam::Geom geo = sam::make_geom(s, 15);
+    const sam::Geom geo = sam::make_geom(s, items_of(dtype));
     const uint64_t h = g % (uint64_t)s;
     const size_t tiles = (size_t)((h + n + geo.T - 1) / geo.T);
     Workspace* ws = nullptr;
     int dev = 0;
-    int rc = get_ws(st, tiles, tiles * (size_t)s * (size_t)k * w, &ws, &dev);
+    int rc = get_ws(st, carry_bytes(dtype, k, s, tiles), &ws, &dev);
     if (rc != SAM_OK) return rc;
     sam::LaunchArgs a;
     a.in = in;
@@ -168,12 +168,10 @@ int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void*
     a.inclusive = inclusive ? 1 : 0;
     a.store_mode = store_mode;
     a.stream = st;
-    a.status = ws->status;
-    a.aggv = ws->aggv;
-    a.inclv = ws->inclv;
+    a.carry = ws->carry;
     a.tile_ctr = (unsigned long long*)(ws->ctr);
     a.done_ctr = (unsigned int*)(ws->ctr + 8);
-    a.epoch_ptr = (unsigned long long*)(ws->ctr + 16);
+    a.epoch_ptr = (unsigned int*)(ws->ctr + 12);
     a.num_sms = num_sms(dev);
     cudaError_t e;
     switch (dtype) {
@@ -232,11 +230,11 @@ int sam_scan_seeded(sam_dtype dtype, int order, int tuple, int inclusive, const 
 int sam_prepare(sam_dtype dtype, int order, int tuple, uint64_t max_n, sam_stream_t stream) {
     int rc = validate_common(dtype, order, tuple);
     if (rc) return rc;
-    const sam::Geom geo = sam::make_geom(tuple, 15);
+    const sam::Geom geo = sam::make_geom(tuple, items_of(dtype));
     const size_t tiles = (size_t)((max_n + tuple + geo.T - 1) / geo.T);
     Workspace* ws = nullptr;
     int dev = 0;
-    return get_ws((cudaStream_t)stream, tiles, tiles * (size_t)tuple * (size_t)order * elem_size(dtype), &ws, &dev);
+    return get_ws((cudaStream_t)stream, carry_bytes(dtype, order, tuple, tiles), &ws, &dev);
 }
 
 size_t sam_shard_payload_bytes(sam_dtype dtype, int order, int tuple) {
@@ -275,7 +273,7 @@ int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const v
     if (rank > 0) {
         Workspace* ws = nullptr;
         int dev = 0;
-        rc = get_ws(st, 0, 0, &ws, &dev);
+        rc = get_ws(st, 0, &ws, &dev);
         if (rc) return rc;
         void* seedbuf = ws->ctr + 32;
         const size_t pb = sam_shard_payload_bytes(dtype, order, tuple);
@@ -414,9 +412,7 @@ int sam_release_workspaces(void) {
     cudaDeviceSynchronize();
     for (auto& kv : g_ws) {
         Workspace* ws = kv.second;
-        if (ws->status) cudaFree(ws->status);
-        if (ws->aggv) cudaFree(ws->aggv);
-        if (ws->inclv) cudaFree(ws->inclv);
+        if (ws->carry) cudaFree(ws->carry);
         if (ws->ctr) cudaFree(ws->ctr);
         delete ws;
     }

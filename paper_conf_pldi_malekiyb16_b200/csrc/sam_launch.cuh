@@ -56,12 +56,10 @@ struct LaunchArgs {
     int store_mode;
     cudaStream_t stream;
     // workspace
-    uint64_t* status;
-    void* aggv;
-    void* inclv;
+    unsigned long long* carry;
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
-    unsigned long long* epoch_ptr;
+    unsigned int* epoch_ptr;
     int num_sms;
 };
 
@@ -115,27 +113,26 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
             if (le >= (int64_t)p.h && le >= 0) p.last_e[m] = le;
         }
     }
-    p.status = a.status;
-    p.aggv = (T*)a.aggv;
-    p.inclv = (T*)a.inclv;
+    p.carry = a.carry;
     p.tile_ctr = a.tile_ctr;
     p.done_ctr = a.done_ctr;
     p.epoch_ptr = a.epoch_ptr;
     mcol<T>(Cfg<T>::ITEMS, K, p.bc);
     mcol<T>(geo.Uw, K, p.bw);
     mcol<T>(geo.U, K, p.bu);
-    mcol<T>((int64_t)geo.Wn * geo.U, K, p.bwin);
+    constexpr int V = LB<T, K>::V;
+    mcol<T>((int64_t)geo.Wn * V * geo.U, K, p.bwin);
     for (int v = 0; v < 32; ++v) {
         T b[K];
         mcol<T>((int64_t)v * Cfg<T>::ITEMS, K, b);
         for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
     }
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
-    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
+    for (int j = 0; j < MAX_LB; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
 
-    uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
-    if (grid > p.num_tiles) grid = p.num_tiles;
-    if (grid < 1) grid = 1;
+    // one CTA per tile (the hardware block scheduler keeps max_blocks_per_sm CTAs per SM busy)
+    const uint64_t grid = p.num_tiles;
+    if (grid == 0 || grid > 0x7fffffffull) return cudaErrorInvalidValue;
     sam_scan_kernel<T, K><<<(unsigned)grid, geo.W * 32, S::BYTES, a.stream>>>(p);
     if (launches) ++*launches;
     return cudaGetLastError();
