@@ -130,10 +130,11 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
     for (int j = 0; j < MAX_LB; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
 
-    // one CTA per tile (the hardware block scheduler keeps max_blocks_per_sm CTAs per SM busy)
-    const uint64_t grid = p.num_tiles;
-    if (grid == 0 || grid > 0x7fffffffull) return cudaErrorInvalidValue;
-    sam_scan_kernel<T, K><<<(unsigned)grid, geo.W * 32, S::BYTES, a.stream>>>(p);
+    // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer + carry warp)
+    uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
+    if (grid > p.num_tiles) grid = p.num_tiles;
+    if (grid < 1) grid = 1;
+    sam_scan_kernel<T, K><<<(unsigned)grid, (geo.W + 2) * 32, S::BYTES, a.stream>>>(p);
     if (launches) ++*launches;
     return cudaGetLastError();
 }

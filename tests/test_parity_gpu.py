@@ -66,15 +66,22 @@ def test_deep_lookback_many_tiles(name, k, s):
         compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
 
 
-@pytest.mark.parametrize("k,s", [(1, 1), (3, 2), (8, 8), (2, 5)])
-def test_edge_sizes(k, s):
-    import paper_conf_pldi_malekiyb16_b200._build as B  # noqa: F401  (library must be there)
+def tile_elems(s, items):
+    """Tile size of the kernel geometry: W*32*items, W = s' * c."""
+    G = s & -s
+    sp = s // G
+    c = max(1, 8 // sp)
+    while c & (c - 1):
+        c &= c - 1
+    return sp * c * 32 * items
 
-    tiles = {1: 3840, 2: 3840, 3: 2880, 4: 3840, 5: 2400, 6: 2880, 7: 3360, 8: 3840}
-    T = tiles[s]
-    for n in sorted({1, 2, 3, s - 1 if s > 1 else 1, s, s + 1, 31, 32, 33, T - 1, T, T + 1, 2 * T - 1,
-                     2 * T + 3, 3 * T + 5}):
-        for name in ("i32", "i64"):
+
+@pytest.mark.parametrize("k,s", [(1, 1), (3, 2), (8, 8), (2, 5), (4, 3), (1, 7)])
+def test_edge_sizes(k, s):
+    for name, items in (("i32", 31), ("i64", 15)):
+        T = tile_elems(s, items)
+        for n in sorted({1, 2, 3, s - 1 if s > 1 else 1, s, s + 1, 31, 32, 33, T - 1, T, T + 1, 2 * T - 1,
+                         2 * T + 3, 3 * T + 5, 7 * T + s}):
             x = synth.make(n, name, "uniform", seed=n)
             for inclusive in (True, False):
                 compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
