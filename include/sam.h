@@ -134,6 +134,11 @@ const char* sam_version(void);
 int sam_release_workspaces(void);
 /* Kernel launches issued by this library on the calling process since load (for bench). */
 uint64_t sam_launch_count(void);
+/* Diagnostics: when trace_dev (device memory, >= 8 * tiles u64) is non-NULL, subsequent scan
+ * launches record %globaltimer at 8 pipeline events of every tile: [tile][claim, P1 start,
+ * P1 done, aggregate published, look-back start, inclusive published, carry applied, stored].
+ * NULL turns tracing off. */
+int sam_debug_set_trace(void* trace_dev);
 
 #ifdef __cplusplus
 }

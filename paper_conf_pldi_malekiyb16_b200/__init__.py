@@ -56,6 +56,7 @@ def lib() -> ctypes.CDLL:
             "sam_version": (ctypes.c_char_p, []),
             "sam_release_workspaces": (I, []),
             "sam_launch_count": (U64, []),
+            "sam_debug_set_trace": (I, [P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)

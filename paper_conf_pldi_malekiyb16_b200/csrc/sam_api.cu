@@ -69,6 +69,7 @@ struct Workspace {
 std::mutex g_mu;
 std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
 std::map<int, int> g_sms;
+unsigned long long* g_trace = nullptr;  // diagnostics: per-tile event timestamps of the next launches
 
 int num_sms(int dev) {
     auto it = g_sms.find(dev);
@@ -173,6 +174,7 @@ int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void*
     a.done_ctr = (unsigned int*)(ws->ctr + 8);
     a.epoch_ptr = (unsigned int*)(ws->ctr + 12);
     a.num_sms = num_sms(dev);
+    a.trace = g_trace;
     cudaError_t e;
     switch (dtype) {
         case SAM_I32: e = dispatch_k<uint32_t>(k, a); break;
@@ -400,6 +402,11 @@ int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const vo
     cudaError_t e = cudaStreamSynchronize(P->s_d2h);
     if (e == cudaSuccess) e = cudaStreamSynchronize(P->s_cmp);
     if (e != cudaSuccess) return cuda_fail(e, "host pipeline");
+    return SAM_OK;
+}
+
+int sam_debug_set_trace(void* trace_dev) {
+    g_trace = (unsigned long long*)trace_dev;
     return SAM_OK;
 }
 

@@ -29,7 +29,7 @@
 //                  scans of the next tiles.  Every published 64-bit word carries the launch's
 //                  32-bit epoch tag beside (half) a value, so each word validates itself: the
 //                  paper's "local sum -> fence -> ready flag" becomes one store with
-//                  no fence, and a look-back hop is ONE L2 round trip over a window of up to 128
+//                  no fence, and a look-back hop is ONE L2 round trip over a window of up to 256
 //                  predecessor tiles; it folds aggregates with the carry operator (M(L) s + v)
 //                  back to the nearest inclusive state -- the O(n) scheme the paper describes for
 //                  CUB and advises once the architectural factor grows
@@ -53,19 +53,21 @@ template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB = 6, LAG 
 template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB = 6, LAG = 2; };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int MAX_THREADS = (MAX_CWARPS + 2) * 32; // + producer warp + carry warp
-constexpr int MAX_LB = 128;                        // max predecessor tiles per look-back round trip
+constexpr int NCARRY = 2;                          // carry (look-back) warps, alternating tiles
+constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
+constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
+constexpr int MAX_LB = 256;                        // max predecessor tiles per look-back round trip
 constexpr int TILE_THREADS = MAX_CWARPS * 32;
 
 enum StoreMode { STORE_BULK = 0, STORE_STRIPED = 1, STORE_NONE = 2 };
 
 // 64-bit tagged words per value: 1 for 32-bit types ([tag|value]), 2 for 64-bit ([tag|lo],[tag|hi])
 template <typename T> struct TagW { static constexpr int W = sizeof(T) == 4 ? 1 : 2; };
-// look-back windows per round trip (carry-warp register budget: V*K*2W <= 32 words per lane)
+// look-back windows per round trip (carry-warp register budget: V*K*2W <= 64 words per lane)
 template <typename T, int K> struct LB {
     static constexpr int W2 = 2 * TagW<T>::W;
-    static constexpr int V0 = 32 / (K * W2);
-    static constexpr int V = V0 < 1 ? 1 : (V0 > 4 ? 4 : V0);
+    static constexpr int V0 = 64 / (K * W2);
+    static constexpr int V = V0 < 1 ? 1 : (V0 > 8 ? 8 : V0);
 };
 
 template <typename T, int K>
@@ -87,6 +89,7 @@ struct Params {
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
+    unsigned long long* trace;  // optional per-tile event timestamps [tile][8] (diagnostics), or null
     T bc[K];              // b_d(ITEMS)
     T bw[K];              // b_d(Uw)
     T bu[K];              // b_d(U)
@@ -114,6 +117,14 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 }
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n}" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
@@ -145,6 +156,16 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// diagnostics: record event ev (0..7) of tile `tile` when tracing is on
+#define SAM_TRACE(ev, tile)                                                        \
+    do {                                                                           \
+        if (p.trace) p.trace[(size_t)(tile) * 8 + (ev)] = globaltimer();           \
+    } while (0)
 __device__ __forceinline__ uint64_t policy_evict_first() {
     uint64_t p;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -215,9 +236,9 @@ struct Smem {
     static constexpr int WQ = 64 * K;             // per-buffer warp states   [64][K]
     static constexpr int LA = 8 * K;              // per-buffer tile aggregate [8][K]
     static constexpr int OFF_BUF = 0;
-    static constexpr int OFF_BAR = OFF_BUF + NB * BUFB;                  // 4 x NB mbarriers
-    static constexpr int OFF_TILE = OFF_BAR + 4 * NB * 8;                // NB x i64
-    static constexpr int OFF_TAG = OFF_TILE + NB * 8;                    // u32
+    static constexpr int OFF_BAR = OFF_BUF + NB * BUFB;                  // 5 x NB mbarriers
+    static constexpr int OFF_TILE = OFF_BAR + 5 * NB * 8;                // NB x i64
+    static constexpr int OFF_TAG = OFF_TILE + NB * 8;                    // u32 tag, i32 end iteration
     static constexpr int OFF_WQ = (OFF_TAG + 8 + 15) / 16 * 16;          // NB x [64][K]
     static constexpr int OFF_LA = OFF_WQ + NB * WQ * (int)sizeof(T);     // NB x [8][K]
     static constexpr int OFF_BT = OFF_LA + NB * LA * (int)sizeof(T);     // [K][32]
@@ -247,8 +268,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint64_t* bar_agg = bar_full + NB;
     uint64_t* bar_carry = bar_agg + NB;
     uint64_t* bar_stored = bar_carry + NB;
+    uint64_t* bar_p1 = bar_stored + NB;
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
     uint32_t* sm_tag = (uint32_t*)(smem + S::OFF_TAG);
+    volatile int* sm_end = (volatile int*)(smem + S::OFF_TAG + 4);
     T* wq_all = (T*)(smem + S::OFF_WQ);
     T* la_all = (T*)(smem + S::OFF_LA);
     T* bt_s = (T*)(smem + S::OFF_BT);
@@ -270,9 +293,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             mbar_init(&bar_agg[b], 32);
             mbar_init(&bar_carry[b], 32);
             mbar_init(&bar_stored[b], NCT);
+            mbar_init(&bar_p1[b], NCT);
         }
         fence_mbar_init();
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
+        *sm_end = -1;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
@@ -306,6 +331,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 if (j >= NB) {  // buffer b last held iteration j-NB: store it, wait for the read
                     const int jo = j - NB;
                     mbar_wait(&bar_stored[b], (uint32_t)((jo / NB) & 1));
+                    if (tile_of[b] >= 0) SAM_TRACE(7, tile_of[b]);
                     store_tile(b);
                     bulk_wait_read0();
                 }
@@ -316,6 +342,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     break;
                 }
                 tile_of[b] = (int64_t)t;
+                SAM_TRACE(0, t);
                 const uint64_t e0 = t * (uint64_t)Tt;
                 const uint64_t lo = e0 > p.h ? e0 : p.h;
                 const uint64_t hi = (e0 + Tt < p.h + p.n) ? e0 + Tt : p.h + p.n;
@@ -337,13 +364,74 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             bulk_wait_all0();
         }
     } else if (warp == NW + 1) {
-        // =========================== carry warp: look-back, inclusive states ====================
+        // =========================== aggregator warp: block combine, aggregate publish ===========
         const int npair = s * c;
         for (int i = 0;; ++i) {
             const int b = i % NB;
-            mbar_wait(&bar_agg[b], (uint32_t)((i / NB) & 1));
+            mbar_wait(&bar_full[b], (uint32_t)((i / NB) & 1));
             const int64_t tile = tile_of[b];
-            if (tile < 0) break;
+            if (tile < 0) {  // end of stream: the carry warps poll this marker while they wait
+                if (lane == 0) *sm_end = i;
+                break;
+            }
+            mbar_wait(&bar_p1[b], (uint32_t)((i / NB) & 1));
+            if (lane == 0) SAM_TRACE(2, tile);
+            T* wq = wq_all + b * S::WQ;
+            T* la = la_all + b * S::LA;
+            for (int pair = lane; pair < 64; pair += 32) {
+                const bool ok = pair < npair;
+                const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
+                T E[K], yl[K];
+#pragma unroll
+                for (int t = 0; t < K; ++t) {
+                    T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
+#pragma unroll
+                    for (int j = 0; j < t; ++j) z += p.bw[t - j] * E[j];
+                    T y = z;
+                    for (int off = 1; off < c; off <<= 1) {
+                        T o = shfl_up(y, off);
+                        if (qq >= off) y += o;
+                    }
+                    if constexpr (IsInt<T>::value) {
+                        E[t] = y - z;
+                    } else {
+                        T o = shfl_up(y, 1);
+                        E[t] = (qq >= 1) ? o : T(0);
+                    }
+                    yl[t] = y;
+                }
+                __syncwarp();
+                if (ok) {
+#pragma unroll
+                    for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = E[t];  // warp-exclusive prefix
+                    if (qq == c - 1) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) {
+                            la[mm * K + t] = yl[t];
+                            if (tile > 0) {  // a4: publish the tile aggregate
+                                put_tagged<T>(p.carry + (((size_t)tile * s + mm) * K + t) * W2, 0, tag, yl[t]);
+                            }
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) SAM_TRACE(3, tile);
+            mbar_arrive(&bar_agg[b]);
+        }
+    } else if (warp >= NW + 2) {
+        // =========================== carry warps: look-back, inclusive states ===================
+        const int npair = s * c;
+        for (int i = warp - (NW + 2);; i += NCARRY) {
+            const int b = i % NB;
+            bool ended = false;
+            while (!mbar_try_wait(&bar_agg[b], (uint32_t)((i / NB) & 1))) {
+                const int end = *sm_end;
+                if (end >= 0 && i >= end) { ended = true; break; }
+            }
+            if (__any_sync(0xffffffffu, ended)) break;
+            const int64_t tile = tile_of[b];
+            if (lane == 0) SAM_TRACE(4, tile);
             T* wq = wq_all + b * S::WQ;
             const T* la = la_all + b * S::LA;
             const bool lane_ok = lane < s;
@@ -537,6 +625,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                 }
             }
+            __syncwarp();
+            if (lane == 0) SAM_TRACE(5, tile);
             mbar_arrive(&bar_carry[b]);
         }
     } else {
@@ -552,6 +642,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         auto carry_apply = [&](int it, int64_t tile, const T* e) {
             const int b = it % NB;
             mbar_wait(&bar_carry[b], (uint32_t)((it / NB) & 1));
+            if (tid == 0) SAM_TRACE(6, tile);
             T* xs = (T*)(smem + S::OFF_BUF + b * S::BUFB + p.delta);
             const T* wq = wq_all + b * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
@@ -668,10 +759,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const int b = i % NB;
             mbar_wait(&bar_full[b], (uint32_t)((i / NB) & 1));
             const int64_t tile = tile_of[b];
-            if (tile < 0) {
-                if (warp == 0) mbar_arrive(&bar_agg[b]);  // lets the carry warp see the end
-                break;
-            }
+            if (tile < 0) break;
+            if (tid == 0) SAM_TRACE(1, tile);
             T* xs = (T*)(smem + S::OFF_BUF + b * S::BUFB + p.delta);
             T* wq = wq_all + b * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
@@ -722,51 +811,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
                 if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
             }
-            named_bar_sync(1, NCT);
-
-            // ---- a3/a4: compute warp 0 combines warp states and publishes the aggregate -----
-            if (warp == 0) {
-                const int npair = s * c;
-                T* la = la_all + b * S::LA;
-                for (int pair = lane; pair < 64; pair += 32) {
-                    const bool ok = pair < npair;
-                    const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
-                    T E[K], yl[K];
-#pragma unroll
-                    for (int t = 0; t < K; ++t) {
-                        T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
-#pragma unroll
-                        for (int j = 0; j < t; ++j) z += p.bw[t - j] * E[j];
-                        T y = z;
-                        for (int off = 1; off < c; off <<= 1) {
-                            T o = shfl_up(y, off);
-                            if (qq >= off) y += o;
-                        }
-                        if constexpr (IsInt<T>::value) {
-                            E[t] = y - z;
-                        } else {
-                            T o = shfl_up(y, 1);
-                            E[t] = (qq >= 1) ? o : T(0);
-                        }
-                        yl[t] = y;
-                    }
-                    __syncwarp();
-                    if (ok) {
-#pragma unroll
-                        for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = E[t];  // warp-exclusive prefix
-                        if (qq == c - 1) {
-#pragma unroll
-                            for (int t = 0; t < K; ++t) {
-                                la[mm * K + t] = yl[t];
-                                if (tile > 0) {
-                                    put_tagged<T>(p.carry + (((size_t)tile * s + mm) * K + t) * W2, 0, tag, yl[t]);
-                                }
-                            }
-                        }
-                    }
-                }
-                mbar_arrive(&bar_agg[b]);
-            }
+            mbar_arrive(&bar_p1[b]);  // warp states ready for the aggregator warp
 
             // ---- a6 for the tile LAG iterations back ------------------------------------------
             if (i >= LAG) carry_apply(i - LAG, tq[0], eq[0]);

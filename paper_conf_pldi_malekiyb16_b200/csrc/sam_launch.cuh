@@ -60,6 +60,7 @@ struct LaunchArgs {
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
+    unsigned long long* trace;
     int num_sms;
 };
 
@@ -117,6 +118,7 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     p.tile_ctr = a.tile_ctr;
     p.done_ctr = a.done_ctr;
     p.epoch_ptr = a.epoch_ptr;
+    p.trace = a.trace;
     mcol<T>(Cfg<T>::ITEMS, K, p.bc);
     mcol<T>(geo.Uw, K, p.bw);
     mcol<T>(geo.U, K, p.bu);
@@ -130,11 +132,11 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
     for (int j = 0; j < MAX_LB; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
 
-    // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer + carry warp)
+    // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
     if (grid > p.num_tiles) grid = p.num_tiles;
     if (grid < 1) grid = 1;
-    sam_scan_kernel<T, K><<<(unsigned)grid, (geo.W + 2) * 32, S::BYTES, a.stream>>>(p);
+    sam_scan_kernel<T, K><<<(unsigned)grid, (geo.W + SERVICE_WARPS) * 32, S::BYTES, a.stream>>>(p);
     if (launches) ++*launches;
     return cudaGetLastError();
 }
