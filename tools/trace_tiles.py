@@ -1,0 +1,28 @@
+"""Per-tile pipeline event trace (developer tool): python tools/trace_tiles.py i32 28 1 1"""
+import sys, os, ctypes
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch, synth
+import paper_conf_pldi_malekiyb16_b200 as S
+dt, logn, k, s = sys.argv[1], int(sys.argv[2]), int(sys.argv[3]), int(sys.argv[4])
+n = 1 << logn
+x = synth.make_torch(n, dt, "uniform", device="cuda"); y = torch.empty_like(x)
+for _ in range(3): S.scan(x, k, s, True, out=y)
+torch.cuda.synchronize()
+tr = torch.zeros(8 * (n // 1000 + 16), dtype=torch.int64, device="cuda")
+S.lib().sam_debug_set_trace(ctypes.c_void_p(tr.data_ptr()))
+S.scan(x, k, s, True, out=y); torch.cuda.synchronize()
+S.lib().sam_debug_set_trace(None)
+t = tr.cpu().numpy().reshape(-1, 8)
+t = t[t[:, 0] > 0]
+t = t - t[:, 0].min()
+names = ["claim", "p1start", "p1done", "aggpub", "lbstart", "inclpub", "p2start", "stored"]
+print(f"{dt} 2^{logn} k={k} s={s}: tiles {len(t)}  span {t.max()/1e3:.1f} us  rate {len(t)/(t.max()/1e3):.1f} tiles/us")
+def q(a): return " ".join(f"{np.percentile(a, pp):7.2f}" for pp in (10, 50, 90, 99))
+print("interval (us)            p10     p50     p90     p99")
+for a_, b_ in [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5), (5, 6), (6, 7), (0, 3), (3, 5), (0, 7)]:
+    d = (t[:, b_] - t[:, a_]) / 1e3
+    print(f"{names[a_]:>8} -> {names[b_]:<8} {q(d)}")
+d = (t[:-1, 3] - t[1:, 3]) / 1e3
+print(f"agg(t-1) - agg(t)        {q(d)}")
+d = (t[:-1, 5] - t[1:, 3]) / 1e3
+print(f"incl(t-1) - agg(t)       {q(d)}")
