@@ -1,39 +1,43 @@
 // sam_kernel.cuh -- single-pass order-k, tuple-s prefix sum for sm_100a.
 //
-// One kernel launch reads every input element once and writes every output element once
-// (P:393-395): SAM's single-pass property, kept for any order and tuple
-// size.  Persistent, warp-specialised CTAs (one per SM) stream tiles of
-// T = W*32*ITEMS elements through a ring of NB shared-memory buffers:
+// One kernel launch reads every input element once from HBM and writes every output element
+// once: SAM's single-pass property, kept for any order and
+// tuple size.  Persistent, warp-specialised CTAs (one per SM) stream tiles of
+// T = W*32*ITEMS elements:
 //
-//   producer warp  a1: claims tiles from an atomic counter, one at a time as buffers free up (so
-//                  a claimed tile's predecessors all belong to running CTAs -- no co-residency
-//                  assumption, cf. P:2475-2479 -- and claims stay interleaved across CTAs), pulls
-//                  each tile into smem with a 1-D cp.async.bulk (TMA bulk engine, mbarrier
-//                  completion) and a7: writes finished tiles back with cp.async.bulk stores.
-//   compute warps  a2: thread <-> (tuple lane m, ITEMS consecutive lane positions), read from
-//                  smem at stride s; a warp holds G = (largest power of two dividing s) lanes,
-//                  32/G threads each, so the strided reads are bank-conflict free (ITEMS odd)
-//                  and registers do not grow with s;
-//                  a3: zero-seeded order-k local scan -- thread-serial recurrence (k adds per
-//                  element), warp scan of thread states (k plain shuffle scans, order by order),
-//                  block combine of warp states: the paper's three-phase intra-block scan
-//                   iterated per order;
-//                  a4: warp 0 publishes the tile's per-lane k-vector aggregate (one value per
-//                  order; all s lanes together) right after the local
-//                  scan -- never behind a look-back;
-//                  a6: LAG tiles later, the fused carry application: thread incoming state =
-//                  M(L) carry + local prefix, then the seeded recurrence produces the outputs
-//                  (the binomial fix-up C(r+t-j, t-j)); exclusive = inclusive shifted by k lane
-//                  positions (R1), the first k from finite differences of the state.
-//   carry warp     a5: decoupled look-back per tile, overlapped with the compute warps' local
-//                  scans of the next tiles.  Every published 64-bit word carries the launch's
-//                  32-bit epoch tag beside (half) a value, so each word validates itself: the
-//                  paper's "local sum -> fence -> ready flag" becomes one store with
-//                  no fence, and a look-back hop is ONE L2 round trip over a window of up to 256
-//                  predecessor tiles; it folds aggregates with the carry operator (M(L) s + v)
-//                  back to the nearest inclusive state -- the O(n) scheme the paper describes for
-//                  CUB and advises once the architectural factor grows
-//                  (B200's af is ~9x the paper's GPUs).
+//   producer warp   a1: claims tiles from an atomic counter, one at a time and at most PF ahead
+//                   of the local scans (every predecessor of a claimed tile belongs to a running
+//                   CTA -- no co-residency assumption), and pulls each tile
+//                   from HBM into a ring of NB1 smem buffers with a 1-D cp.async.bulk (TMA bulk
+//                   engine) marked L2::evict_last.  When the tile's carry is known it pulls the
+//                   same bytes again -- now from the 126 MB L2 (~18 TB/s vs ~7 TB/s HBM) -- into a
+//                   second ring of NB2 buffers, and a7: writes the finished tile back with a
+//                   cp.async.bulk store.  The look-back's latency is spent with the tile parked
+//                   in L2, not in shared memory, so it no longer throttles the HBM stream.
+//   compute warps   a2: thread <-> (tuple lane m, ITEMS consecutive lane positions), read from
+//                   smem at stride s; a warp holds G = (largest power of two dividing s) lanes,
+//                   32/G threads each, so the strided reads are bank-conflict free (ITEMS odd)
+//                   and registers do not grow with s;
+//                   a3: zero-seeded order-k local scan -- thread-serial recurrence (k adds per
+//                   element) and a warp scan of thread states (k plain shuffle scans, order by
+//                   order): the paper's three-phase intra-block scan iterated per
+//                   order;
+//                   a6: once the carry is known, the fused carry application: thread incoming
+//                   state = M(L) carry + local prefix, then the seeded recurrence produces the
+//                   outputs (the binomial fix-up C(r+t-j, t-j)); exclusive = inclusive shifted by
+//                   k lane positions (R1), the first k from finite differences.
+//                   A loaded tile's local scan always goes first (its aggregate gates other
+//                   CTAs' look-backs); up to LAG tiles may await their carries.
+//   aggregator warp a3/a4: combines the warp states of a tile and publishes its per-lane k-vector
+//                   aggregate (one value per order; all s lanes).
+//   carry warps     a5: decoupled look-back.  Every published 64-bit word carries the launch's
+//                   32-bit epoch tag beside (half) a value, so each word validates itself: the
+//                   paper's "local sum -> fence -> ready flag" becomes one store with
+//                   no fence, and a look-back hop is ONE L2 round trip over a window of up to 512
+//                   predecessor tiles, folded with the carry operator (M(L) s + v) back to the
+//                   nearest inclusive state -- the O(n) scheme the paper describes for CUB
+//                    and advises once the architectural factor grows (
+//                   B200's af is ~9x the paper's GPUs).
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -45,29 +49,29 @@
 namespace sam {
 
 template <typename T> struct Cfg;
-// ITEMS odd (bank-conflict-free strided smem reads); NB smem tile buffers; LAG = tiles between a
-// tile's local scan and its carry application (the look-back's latency budget).
-template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31, NB = 6, LAG = 2; };
-template <> struct Cfg<float>    { static constexpr int ITEMS = 31, NB = 6, LAG = 2; };
-template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB = 6, LAG = 2; };
-template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB = 6, LAG = 2; };
+// ITEMS odd (bank-conflict-free strided smem reads); NB1 / NB2 smem buffers for local scans / carry
+// application + store; LAG = max tiles between local scan and carry application (the look-back's
+// latency budget, states in registers); PF = max claimed-but-unscanned tiles per CTA.
+template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
+template <> struct Cfg<float>    { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
+template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
+template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int NCARRY = 2;                          // carry (look-back) warps, alternating tiles
+constexpr int NCARRY = 3;                          // carry (look-back) warps, round-robin over tiles
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
-constexpr int MAX_LB = 256;                        // max predecessor tiles per look-back round trip
 constexpr int TILE_THREADS = MAX_CWARPS * 32;
 
 enum StoreMode { STORE_BULK = 0, STORE_STRIPED = 1, STORE_NONE = 2 };
 
 // 64-bit tagged words per value: 1 for 32-bit types ([tag|value]), 2 for 64-bit ([tag|lo],[tag|hi])
 template <typename T> struct TagW { static constexpr int W = sizeof(T) == 4 ? 1 : 2; };
-// look-back windows per round trip (carry-warp register budget: V*K*2W <= 64 words per lane)
+// look-back window rows per round trip (carry-warp register budget: V*K*2W <= 16 words per lane)
 template <typename T, int K> struct LB {
     static constexpr int W2 = 2 * TagW<T>::W;
-    static constexpr int V0 = 64 / (K * W2);
-    static constexpr int V = V0 < 1 ? 1 : (V0 > 8 ? 8 : V0);
+    static constexpr int V0 = 16 / (K * W2);
+    static constexpr int V = V0 < 1 ? 1 : (V0 > 16 ? 16 : V0);
 };
 
 template <typename T, int K>
@@ -94,9 +98,10 @@ struct Params {
     T bw[K];              // b_d(Uw)
     T bu[K];              // b_d(U)
     T bwin[K];            // b_d(Wn*V*U)   (one look-back round trip further)
+    T bwn[K];             // b_d(Wn*U)     (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bq[8][K];           // b_d(q*Uw),     q < c
-    T bl[MAX_LB][K];      // b_d(d*U),      d < Wn*V
+    T bl[32][K];          // b_d(j*U),      j < Wn
 };
 
 // ------------------------------------------------------------------------------------------
@@ -147,6 +152,10 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
 __device__ __forceinline__ void bulk_wait_all0() {
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
@@ -166,6 +175,11 @@ __device__ __forceinline__ unsigned long long globaltimer() {
     do {                                                                           \
         if (p.trace) p.trace[(size_t)(tile) * 8 + (ev)] = globaltimer();           \
     } while (0)
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
 __device__ __forceinline__ uint64_t policy_evict_first() {
     uint64_t p;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -229,19 +243,24 @@ template <> struct IsInt<uint64_t> { static constexpr bool value = true; };
 template <typename T, int K>
 struct Smem {
     static constexpr int ITEMS = Cfg<T>::ITEMS;
-    static constexpr int NB = Cfg<T>::NB;
+    static constexpr int NB1 = Cfg<T>::NB1;
+    static constexpr int NB2 = Cfg<T>::NB2;
+    static constexpr int LAG = Cfg<T>::LAG;
+    static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
     static constexpr int TMAX = TILE_THREADS * ITEMS;
-    static constexpr int NBL = 32 * LB<T, K>::V;  // look-back binomial rows
+    static constexpr int NBL = 32;                // look-back binomial rows
     static constexpr int BUFB = ((TMAX * (int)sizeof(T) + 32) + 127) / 128 * 128;
-    static constexpr int WQ = 64 * K;             // per-buffer warp states   [64][K]
-    static constexpr int LA = 8 * K;              // per-buffer tile aggregate [8][K]
-    static constexpr int OFF_BUF = 0;
-    static constexpr int OFF_BAR = OFF_BUF + NB * BUFB;                  // 5 x NB mbarriers
-    static constexpr int OFF_TILE = OFF_BAR + 5 * NB * 8;                // NB x i64
-    static constexpr int OFF_TAG = OFF_TILE + NB * 8;                    // u32 tag, i32 end iteration
-    static constexpr int OFF_WQ = (OFF_TAG + 8 + 15) / 16 * 16;          // NB x [64][K]
-    static constexpr int OFF_LA = OFF_WQ + NB * WQ * (int)sizeof(T);     // NB x [8][K]
-    static constexpr int OFF_BT = OFF_LA + NB * LA * (int)sizeof(T);     // [K][32]
+    static constexpr int WQ = 64 * K;             // per-iteration warp states   [64][K]
+    static constexpr int LA = 8 * K;              // per-iteration tile aggregate [8][K]
+    static constexpr int OFF_BUF1 = 0;
+    static constexpr int OFF_BUF2 = OFF_BUF1 + NB1 * BUFB;
+    static constexpr int OFF_BAR = OFF_BUF2 + NB2 * BUFB;  // full1[NB1] full2[NB2] stored2[NB2] p1/agg/carry[NQ]
+    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ;
+    static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
+    static constexpr int OFF_TAG = OFF_TILE + NQ * 8;                    // u32 tag, i32 end iteration
+    static constexpr int OFF_WQ = (OFF_TAG + 8 + 15) / 16 * 16;          // NQ x [64][K]
+    static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
+    static constexpr int OFF_BT = OFF_LA + NQ * LA * (int)sizeof(T);     // [K][32]
     static constexpr int OFF_BL = OFF_BT + K * 32 * (int)sizeof(T);      // [NBL][K]
     static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
     static constexpr int BYTES = OFF_BQ + 8 * K * (int)sizeof(T);
@@ -255,20 +274,24 @@ __global__ void __launch_bounds__(MAX_THREADS, 1)
 sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     using S = Smem<T, K>;
     constexpr int ITEMS = S::ITEMS;
-    constexpr int NB = S::NB;
+    constexpr int NB1 = S::NB1;
+    constexpr int NB2 = S::NB2;
+    constexpr int NQ = S::NQ;
     constexpr int LAG = Cfg<T>::LAG;
+    constexpr int PF = Cfg<T>::PF;
     constexpr int W2 = 2 * TagW<T>::W;  // tagged words per slot (aggregate + inclusive)
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
-    static_assert(NB >= LAG + 3, "ring: LAG+1 tiles awaiting carries, one storing, one loading");
+    static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 3, "ring sizes");
 
     extern __shared__ __align__(128) unsigned char smem[];
-    uint64_t* bar_full = (uint64_t*)(smem + S::OFF_BAR);
-    uint64_t* bar_agg = bar_full + NB;
-    uint64_t* bar_carry = bar_agg + NB;
-    uint64_t* bar_stored = bar_carry + NB;
-    uint64_t* bar_p1 = bar_stored + NB;
+    uint64_t* bar_full1 = (uint64_t*)(smem + S::OFF_BAR);
+    uint64_t* bar_full2 = bar_full1 + NB1;
+    uint64_t* bar_stored2 = bar_full2 + NB2;
+    uint64_t* bar_p1 = bar_stored2 + NB2;
+    uint64_t* bar_agg = bar_p1 + NQ;
+    uint64_t* bar_carry = bar_agg + NQ;
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
     uint32_t* sm_tag = (uint32_t*)(smem + S::OFF_TAG);
     volatile int* sm_end = (volatile int*)(smem + S::OFF_TAG + 4);
@@ -284,16 +307,18 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     const int NW = p.W;          // compute warps
     const int NCT = NW * 32;     // compute threads
     const int Tt = p.T_;
-    const uint64_t pol = policy_evict_first();
 
     // ---- prologue: barriers, tables, epoch tag -------------------------------------------------
     if (tid == 0) {
-        for (int b = 0; b < NB; ++b) {
-            mbar_init(&bar_full[b], 1);
-            mbar_init(&bar_agg[b], 32);
-            mbar_init(&bar_carry[b], 32);
-            mbar_init(&bar_stored[b], NCT);
-            mbar_init(&bar_p1[b], NCT);
+        for (int b = 0; b < NB1; ++b) mbar_init(&bar_full1[b], 1);
+        for (int b = 0; b < NB2; ++b) {
+            mbar_init(&bar_full2[b], 1);
+            mbar_init(&bar_stored2[b], NCT);
+        }
+        for (int q = 0; q < NQ; ++q) {
+            mbar_init(&bar_p1[q], NCT);
+            mbar_init(&bar_agg[q], 32);
+            mbar_init(&bar_carry[q], 32);
         }
         fence_mbar_init();
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
@@ -305,61 +330,93 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     __syncthreads();
     const uint32_t tag = *sm_tag;
 
+    // wait for barrier phase `par`, or return false once the stream has ended before iteration it
+    auto wait_or_end = [&](uint64_t* bar, uint32_t par, int it) -> bool {
+        bool ended = false;
+        while (!mbar_try_wait(bar, par)) {
+            const int end = *sm_end;
+            if (end >= 0 && it >= end) { ended = true; break; }
+        }
+        return !__any_sync(0xffffffffu, ended);
+    };
+
     if (warp == NW) {
-        // =========================== producer warp: claims, loads, stores ======================
+        // =========================== producer warp: claims, loads, reloads, stores =============
         if (lane == 0) {
-            auto store_tile = [&](int b) {
-                const int64_t tile = tile_of[b];
-                if (p.store_mode != STORE_BULK || tile < 0) return;
+            const uint64_t pol_keep = policy_evict_last();
+            const uint64_t pol_stream = policy_evict_first();
+            auto tile_range = [&](int64_t tile, uint64_t& lo, uint64_t& hi) {
                 const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
-                const uint64_t lo = e0 > p.h ? e0 : p.h;
-                const uint64_t hi = (e0 + Tt < p.h + p.n) ? e0 + Tt : p.h + p.n;
+                lo = e0 > p.h ? e0 : p.h;
+                hi = (e0 + Tt < p.h + p.n) ? e0 + Tt : p.h + p.n;
+            };
+            auto load_tile = [&](int64_t tile, unsigned char* buf, uint64_t* bar, uint64_t pol) {
+                uint64_t lo, hi;
+                tile_range(tile, lo, hi);
+                const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
+                const uintptr_t src_lo = (uintptr_t)p.in + (lo - p.h) * sizeof(T);
+                const uintptr_t src_hi = (uintptr_t)p.in + (hi - p.h) * sizeof(T);
+                const uintptr_t a16 = src_lo & ~(uintptr_t)15;
+                const uintptr_t b16 = (src_hi + 15) & ~(uintptr_t)15;
+                unsigned char* dst = buf + p.delta + (lo - e0) * sizeof(T) - (src_lo - a16);
+                mbar_arrive_expect_tx(bar, (uint32_t)(b16 - a16));
+                bulk_g2s(dst, (const void*)a16, (uint32_t)(b16 - a16), bar, pol);
+            };
+            auto store_tile = [&](int64_t tile, const unsigned char* buf) {
+                if (p.store_mode != STORE_BULK) return;
+                uint64_t lo, hi;
+                tile_range(tile, lo, hi);
+                const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
                 const uintptr_t ob = (uintptr_t)p.out + (lo - p.h) * sizeof(T);
                 const uintptr_t oe = (uintptr_t)p.out + (hi - p.h) * sizeof(T);
                 const uintptr_t bs = (ob + 15) & ~(uintptr_t)15;
                 const uintptr_t be = oe & ~(uintptr_t)15;
                 if (be > bs) {
-                    const unsigned char* src =
-                        smem + S::OFF_BUF + b * S::BUFB + p.delta + (lo - e0) * sizeof(T) + (bs - ob);
-                    bulk_s2g((void*)bs, src, (uint32_t)(be - bs), pol);
-                    bulk_commit();
+                    const unsigned char* src = buf + p.delta + (lo - e0) * sizeof(T) + (bs - ob);
+                    bulk_s2g((void*)bs, src, (uint32_t)(be - bs), pol_stream);
                 }
+                bulk_commit();  // one group per stored iteration (possibly empty)
             };
-            int j = 0;
-            for (;; ++j) {
-                const int b = j % NB;
-                if (j >= NB) {  // buffer b last held iteration j-NB: store it, wait for the read
-                    const int jo = j - NB;
-                    mbar_wait(&bar_stored[b], (uint32_t)((jo / NB) & 1));
-                    if (tile_of[b] >= 0) SAM_TRACE(7, tile_of[b]);
-                    store_tile(b);
-                    bulk_wait_read0();
+            int j1 = 0, j2 = 0, j3 = 0, jend = -1;
+            for (;;) {
+                // (1) store the oldest iteration whose carry application is done
+                if (j3 < j2 && mbar_try_wait(&bar_stored2[j3 % NB2], (uint32_t)((j3 / NB2) & 1))) {
+                    if (p.trace) SAM_TRACE(7, tile_of[j3 % NQ]);
+                    store_tile(tile_of[j3 % NQ], smem + S::OFF_BUF2 + (j3 % NB2) * S::BUFB);
+                    ++j3;
+                    continue;
                 }
-                const unsigned long long t = atomicAdd(p.tile_ctr, 1ull);
-                if (t >= p.num_tiles) {
-                    tile_of[b] = -1;
-                    mbar_arrive(&bar_full[b]);
-                    break;
+                // (2) reload (from L2) the next tile whose carry is known, into a free carry buffer
+                if (j2 < j1 && j2 - j3 < NB2 &&
+                    mbar_try_wait(&bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
+                    // groups committed after the store that last used this buffer (iteration j2-NB2)
+                    const int later = j3 - 1 - (j2 - NB2);
+                    if (later <= 0) bulk_wait_read<0>();
+                    else if (later == 1) bulk_wait_read<1>();
+                    else bulk_wait_read<2>();
+                    load_tile(tile_of[j2 % NQ], smem + S::OFF_BUF2 + (j2 % NB2) * S::BUFB, &bar_full2[j2 % NB2],
+                              pol_stream);
+                    ++j2;
+                    continue;
                 }
-                tile_of[b] = (int64_t)t;
-                SAM_TRACE(0, t);
-                const uint64_t e0 = t * (uint64_t)Tt;
-                const uint64_t lo = e0 > p.h ? e0 : p.h;
-                const uint64_t hi = (e0 + Tt < p.h + p.n) ? e0 + Tt : p.h + p.n;
-                const uintptr_t src_lo = (uintptr_t)p.in + (lo - p.h) * sizeof(T);
-                const uintptr_t src_hi = (uintptr_t)p.in + (hi - p.h) * sizeof(T);
-                const uintptr_t a16 = src_lo & ~(uintptr_t)15;
-                const uintptr_t b16 = (src_hi + 15) & ~(uintptr_t)15;
-                unsigned char* dst =
-                    smem + S::OFF_BUF + b * S::BUFB + p.delta + (lo - e0) * sizeof(T) - (src_lo - a16);
-                mbar_arrive_expect_tx(&bar_full[b], (uint32_t)(b16 - a16));
-                bulk_g2s(dst, (const void*)a16, (uint32_t)(b16 - a16), &bar_full[b], pol);
-            }
-            // drain: iterations loaded but not yet stored
-            for (int jo = (j - NB + 1 > 0 ? j - NB + 1 : 0); jo < j; ++jo) {
-                const int b = jo % NB;
-                mbar_wait(&bar_stored[b], (uint32_t)((jo / NB) & 1));
-                store_tile(b);
+                // (3) claim and load a new tile (buffer free, at most PF unscanned, slot free)
+                if (jend < 0 && j3 > j1 - NQ &&
+                    (j1 < NB1 || mbar_try_wait(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
+                    (j1 < PF || mbar_try_wait(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
+                    const unsigned long long t = atomicAdd(p.tile_ctr, 1ull);
+                    if (t >= p.num_tiles) {
+                        jend = j1;
+                        *sm_end = j1;
+                    } else {
+                        tile_of[j1 % NQ] = (int64_t)t;
+                        SAM_TRACE(0, t);
+                        load_tile((int64_t)t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1],
+                                  pol_keep);
+                        ++j1;
+                    }
+                    continue;
+                }
+                if (jend >= 0 && j3 == jend) break;
             }
             bulk_wait_all0();
         }
@@ -367,17 +424,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // =========================== aggregator warp: block combine, aggregate publish ===========
         const int npair = s * c;
         for (int i = 0;; ++i) {
-            const int b = i % NB;
-            mbar_wait(&bar_full[b], (uint32_t)((i / NB) & 1));
-            const int64_t tile = tile_of[b];
-            if (tile < 0) {  // end of stream: the carry warps poll this marker while they wait
-                if (lane == 0) *sm_end = i;
-                break;
-            }
-            mbar_wait(&bar_p1[b], (uint32_t)((i / NB) & 1));
+            const int qs = i % NQ;
+            if (!wait_or_end(&bar_p1[qs], (uint32_t)((i / NQ) & 1), i)) break;
+            const int64_t tile = tile_of[qs];
             if (lane == 0) SAM_TRACE(2, tile);
-            T* wq = wq_all + b * S::WQ;
-            T* la = la_all + b * S::LA;
+            T* wq = wq_all + qs * S::WQ;
+            T* la = la_all + qs * S::LA;
             for (int pair = lane; pair < 64; pair += 32) {
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
@@ -417,28 +469,20 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             }
             __syncwarp();
             if (lane == 0) SAM_TRACE(3, tile);
-            mbar_arrive(&bar_agg[b]);
+            mbar_arrive(&bar_agg[qs]);
         }
     } else if (warp >= NW + 2) {
-        // =========================== carry warps: look-back, inclusive states ===================
+        // =========================== carry warps: decoupled look-back, inclusive states ==========
         const int npair = s * c;
         for (int i = warp - (NW + 2);; i += NCARRY) {
-            const int b = i % NB;
-            bool ended = false;
-            while (!mbar_try_wait(&bar_agg[b], (uint32_t)((i / NB) & 1))) {
-                const int end = *sm_end;
-                if (end >= 0 && i >= end) { ended = true; break; }
-            }
-            if (__any_sync(0xffffffffu, ended)) break;
-            const int64_t tile = tile_of[b];
+            const int qs = i % NQ;
+            if (!wait_or_end(&bar_agg[qs], (uint32_t)((i / NQ) & 1), i)) break;
+            const int64_t tile = tile_of[qs];
             if (lane == 0) SAM_TRACE(4, tile);
-            T* wq = wq_all + b * S::WQ;
-            const T* la = la_all + b * S::LA;
+            T* wq = wq_all + qs * S::WQ;
+            const T* la = la_all + qs * S::LA;
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
-            T A[K], C[K];
-#pragma unroll
-            for (int t = 0; t < K; ++t) A[t] = la[ml * K + t];
 
             // seed of virtual tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, T* out) {
@@ -454,12 +498,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     for (int t = 0; t < K; ++t) out[t] = T(0);
                 }
             };
-            unsigned long long* const carry_tile = p.carry + (size_t)tile * s * K * W2;
 
+            constexpr int INF = 1 << 30;
+            T C[K];
             if (tile == 0) {
                 seed_of(ml, C);
             } else {
-                // a5: decoupled look-back.  lane = (jl, mlb): predecessor distance d = jl + Wn*vv
+                // a5: lane = (jl, mlb); window row vv holds predecessor distance d = jl + Wn*vv
                 const int Wn = p.Wn;
                 const int jl = lane / s, mlb = lane - jl * s;
                 const bool active = jl < Wn;
@@ -471,7 +516,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 bool first = true;
                 for (;;) {
                     unsigned long long w[V][K][W2];
-                    int st[V];  // 0 invalid, 1 aggregate valid, 2 inclusive valid, 3 beyond the seed
+                    int st[V];  // 0 invalid, 1 aggregate valid, 2 inclusive valid, 3 ignored
 #pragma unroll
                     for (int vv = 0; vv < V; ++vv) {
                         const int64_t idx = basei - jl - (int64_t)Wn * vv;
@@ -503,13 +548,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                 st[vv] = in ? 2 : (ag ? 1 : 0);
                             }
                         }
-                        // nearest predecessor whose s lanes are all inclusive-valid / nearest invalid
-                        dI = 1 << 30;
-                        int dX = 1 << 30;
+                        // nearest tile whose s lanes are all inclusive-valid, nearest invalid one
+                        dI = INF;
+                        int dX = INF;
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
                             const unsigned bv = __ballot_sync(0xffffffffu, st[vv] >= 1);
-                            const unsigned bi = __ballot_sync(0xffffffffu, st[vv] >= 2);
+                            const unsigned bi = __ballot_sync(0xffffffffu, st[vv] == 2);
                             unsigned gv = bv, gi = bi;
                             if (s > 1) {
                                 gv = gi = 0;
@@ -520,20 +565,24 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             }
                             const unsigned full = (Wn == 32) ? 0xffffffffu : ((1u << Wn) - 1u);
                             const unsigned inv = ~gv & full;
-                            if (gi && dI == (1 << 30)) dI = Wn * vv + (__ffs(gi) - 1);
-                            if (inv && dX == (1 << 30)) dX = Wn * vv + (__ffs(inv) - 1);
+                            if (gi && dI == INF) dI = Wn * vv + (__ffs(gi) - 1);
+                            if (inv && dX == INF) dX = Wn * vv + (__ffs(inv) - 1);
                         }
-                        if (dI < dX || (dX == (1 << 30) && dI == (1 << 30))) break;
+                        if (dI < dX || (dX == INF && dI == INF)) break;
                     }
-                    // fold: sum over d <= dI of M(d*U) X_d  (X = inclusive at dI, aggregates before)
+                    // fold: d < dI aggregates, d == dI inclusive.  This lane's tiles sit at
+                    // d = jl + Wn*vv, so by Horner in vv:
+                    //   sum_vv M((jl + Wn vv) U) X_vv = M(jl U) (X_0 + M(Wn U)(X_1 + M(Wn U)(X_2 + ...)))
                     T Y[K];
 #pragma unroll
                     for (int t = 0; t < K; ++t) Y[t] = T(0);
 #pragma unroll
-                    for (int vv = 0; vv < V; ++vv) {
+                    for (int vv = V - 1; vv >= 0; --vv) {
                         const int d = jl + Wn * vv;
+                        T X[K];
+#pragma unroll
+                        for (int t = 0; t < K; ++t) X[t] = T(0);
                         if (active && d <= dI && st[vv] != 3) {
-                            T X[K];
                             const int64_t idx = basei - d;
                             if (idx == -1) {
                                 seed_of(mlb, X);
@@ -549,13 +598,27 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                     }
                                 }
                             }
+                        }
+                        if (vv == V - 1) {
 #pragma unroll
-                            for (int t = 0; t < K; ++t) {
-                                T acc2 = X[t];
+                            for (int t = 0; t < K; ++t) Y[t] = X[t];
+                        } else {
 #pragma unroll
-                                for (int j = 0; j < t; ++j) acc2 += bl_s[d * K + (t - j)] * X[j];
-                                Y[t] += acc2;
+                            for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn U) Y + X
+                                T acc2 = Y[t] + X[t];
+#pragma unroll
+                                for (int j = 0; j < t; ++j) acc2 += p.bwn[t - j] * Y[j];
+                                Y[t] = acc2;
                             }
+                        }
+                    }
+                    if (active) {  // Y <- M(jl U) Y
+#pragma unroll
+                        for (int t = K - 1; t >= 1; --t) {
+                            T acc2 = Y[t];
+#pragma unroll
+                            for (int j = 0; j < t; ++j) acc2 += bl_s[jl * K + (t - j)] * Y[j];
+                            Y[t] = acc2;
                         }
                     }
                     for (int off = 1; off < Wn; off <<= 1) {
@@ -578,7 +641,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             total[t] += acc2;
                         }
                     }
-                    if (dI < (1 << 30)) break;
+                    if (dI < INF) break;
                     {   // Pm <- Pm * M(Wn*V*U)  (truncated polynomial product)
                         T np[K];
 #pragma unroll
@@ -600,9 +663,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 
             // publish the inclusive state of this tile: M(U) C + A
             if ((uint64_t)tile + 1 < p.num_tiles && lane_ok) {
+                unsigned long long* const carry_tile = p.carry + (size_t)tile * s * K * W2;
 #pragma unroll
                 for (int t = 0; t < K; ++t) {
-                    T acc2 = C[t] + A[t];
+                    T acc2 = C[t] + la[ml * K + t];
 #pragma unroll
                     for (int j = 0; j < t; ++j) acc2 += p.bu[t - j] * C[j];
                     put_tagged<T>(carry_tile + (lane * K + t) * W2, 1, tag, acc2);
@@ -627,7 +691,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             }
             __syncwarp();
             if (lane == 0) SAM_TRACE(5, tile);
-            mbar_arrive(&bar_carry[b]);
+            mbar_arrive(&bar_carry[qs]);
         }
     } else {
         // =========================== compute warps ===============================================
@@ -640,11 +704,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 
         // a6 for iteration `it` (tile `tile`, local exclusive state e)
         auto carry_apply = [&](int it, int64_t tile, const T* e) {
-            const int b = it % NB;
-            mbar_wait(&bar_carry[b], (uint32_t)((it / NB) & 1));
+            const int b2 = it % NB2;
+            const int qs = it % NQ;
             if (tid == 0) SAM_TRACE(6, tile);
-            T* xs = (T*)(smem + S::OFF_BUF + b * S::BUFB + p.delta);
-            const T* wq = wq_all + b * S::WQ;
+            T* xs = (T*)(smem + S::OFF_BUF2 + b2 * S::BUFB + p.delta);
+            const T* wq = wq_all + qs * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
             const bool masked = (e0 < p.h) || (e0 + Tt > p.h + p.n);
             T y[K];
@@ -749,87 +813,113 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 named_bar_sync(2, NCT);
                 for (uint64_t ve = lo + tid; ve < hi; ve += NCT) p.out[ve - p.h] = xs[ve - e0];
             }
-            mbar_arrive(&bar_stored[b]);
+            mbar_arrive(&bar_stored2[b2]);
         };
 
+        // Scheduling: a loaded tile's local scan (P1) always goes first, so its aggregate is
+        // published as early as possible (predecessor aggregates gate every look-back); a tile's
+        // carry application (P2) runs once the producer has re-fetched it (its carry is known).
+        // Up to LAG tiles may sit between P1 and P2; their local exclusive states wait in
+        // registers (eq, a static ring indexed by iteration mod LAG).
         T eq[LAG][K];
-        int64_t tq[LAG];
-        int i = 0;
-        for (;; ++i) {
-            const int b = i % NB;
-            mbar_wait(&bar_full[b], (uint32_t)((i / NB) & 1));
-            const int64_t tile = tile_of[b];
-            if (tile < 0) break;
-            if (tid == 0) SAM_TRACE(1, tile);
-            T* xs = (T*)(smem + S::OFF_BUF + b * S::BUFB + p.delta);
-            T* wq = wq_all + b * S::WQ;
-            const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
-            const bool masked = (e0 < p.h) || (e0 + Tt > p.h + p.n);
-
-            // ---- a2/a3: lane run, thread-serial zero-seeded recurrence ----------------------
-            T acc[K];
+        int p1_next = 0, p2_next = 0;
+        for (;;) {
+            const int end = *sm_end;
+            // ---- P1 of the next loaded tile, if the state ring has room ---------------------------
+            if ((end < 0 || p1_next < end) && p1_next < p2_next + LAG) {
+                const int i = p1_next;
+                const int b1 = i % NB1;
+                const uint32_t par = (uint32_t)((i / NB1) & 1);
+                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_try_wait(&bar_full1[b1], par) : 0, 0);
+                if (ready) {
+                    mbar_wait(&bar_full1[b1], par);
+                    const int qs = i % NQ;
+                    const int64_t tile = tile_of[qs];
+                    if (tid == 0) SAM_TRACE(1, tile);
+                    const T* xs = (const T*)(smem + S::OFF_BUF1 + b1 * S::BUFB + p.delta);
+                    T* wq = wq_all + qs * S::WQ;
+                    const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
+                    const bool masked = (e0 < p.h) || (e0 + Tt > p.h + p.n);
+                    // a2/a3: lane run, thread-serial zero-seeded recurrence
+                    T acc[K];
 #pragma unroll
-            for (int t = 0; t < K; ++t) acc[t] = T(0);
-            if (!masked) {
+                    for (int t = 0; t < K; ++t) acc[t] = T(0);
+                    if (!masked) {
 #pragma unroll
-                for (int it = 0; it < ITEMS; ++it) {
-                    const T x = xs[base_loc + it * s];
-                    acc[0] += x;
+                        for (int it = 0; it < ITEMS; ++it) {
+                            const T x = xs[base_loc + it * s];
+                            acc[0] += x;
 #pragma unroll
-                    for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
-                }
-            } else {
+                            for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                        }
+                    } else {
 #pragma unroll
-                for (int it = 0; it < ITEMS; ++it) {
-                    const int el = base_loc + it * s;
-                    const uint64_t ve = e0 + el;
-                    const T x = (ve >= p.h && ve < p.h + p.n) ? xs[el] : T(0);
-                    acc[0] += x;
+                        for (int it = 0; it < ITEMS; ++it) {
+                            const int el = base_loc + it * s;
+                            const uint64_t ve = e0 + el;
+                            const T x = (ve >= p.h && ve < p.h + p.n) ? xs[el] : T(0);
+                            acc[0] += x;
 #pragma unroll
-                    for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                            for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                        }
+                    }
+                    // a3: warp scan of thread states (order by order, plain shuffle scans)
+                    // e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
+                    // z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]
+                    T e[K];
+#pragma unroll
+                    for (int t = 0; t < K; ++t) {
+                        T z = acc[t];
+#pragma unroll
+                        for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
+                        T y = z;
+                        for (int off = G; off < 32; off <<= 1) {
+                            T o = shfl_up(y, off);
+                            if (lane >= off) y += o;
+                        }
+                        if constexpr (IsInt<T>::value) {
+                            e[t] = y - z;
+                        } else {
+                            T o = shfl_up(y, G);
+                            e[t] = (lane >= G) ? o : T(0);
+                        }
+                        if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
+                    }
+                    mbar_arrive(&bar_p1[qs]);  // warp states ready; P1 buffer free for the producer
+#pragma unroll
+                    for (int j = 0; j < LAG; ++j) {
+                        if (j == i % LAG) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) eq[j][t] = e[t];
+                        }
+                    }
+                    ++p1_next;
+                    continue;
                 }
             }
-            // ---- a3: warp scan of thread states (order by order, plain shuffle scans) -------
-            // e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
-            // z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]
-            T e[K];
+            // ---- P2 of the oldest scanned tile once it has been re-fetched with its carry --------
+            if (p2_next < p1_next) {
+                const int i = p2_next;
+                const int b2 = i % NB2;
+                const uint32_t par = (uint32_t)((i / NB2) & 1);
+                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_try_wait(&bar_full2[b2], par) : 0, 0);
+                if (ready) {
+                    mbar_wait(&bar_full2[b2], par);
+                    T e[K];
 #pragma unroll
-            for (int t = 0; t < K; ++t) {
-                T z = acc[t];
+                    for (int j = 0; j < LAG; ++j) {
+                        if (j == i % LAG) {
 #pragma unroll
-                for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
-                T y = z;
-                for (int off = G; off < 32; off <<= 1) {
-                    T o = shfl_up(y, off);
-                    if (lane >= off) y += o;
+                            for (int t = 0; t < K; ++t) e[t] = eq[j][t];
+                        }
+                    }
+                    carry_apply(i, tile_of[i % NQ], e);
+                    ++p2_next;
+                    continue;
                 }
-                if constexpr (IsInt<T>::value) {
-                    e[t] = y - z;
-                } else {
-                    T o = shfl_up(y, G);
-                    e[t] = (lane >= G) ? o : T(0);
-                }
-                if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
+            } else if (end >= 0 && p1_next >= end) {
+                break;
             }
-            mbar_arrive(&bar_p1[b]);  // warp states ready for the aggregator warp
-
-            // ---- a6 for the tile LAG iterations back ------------------------------------------
-            if (i >= LAG) carry_apply(i - LAG, tq[0], eq[0]);
-#pragma unroll
-            for (int j = 0; j + 1 < LAG; ++j) {
-                tq[j] = tq[j + 1];
-#pragma unroll
-                for (int t = 0; t < K; ++t) eq[j][t] = eq[j + 1][t];
-            }
-            tq[LAG - 1] = tile;
-#pragma unroll
-            for (int t = 0; t < K; ++t) eq[LAG - 1][t] = e[t];
-        }
-        // drain the tiles still waiting for their carries
-#pragma unroll
-        for (int j = 0; j < LAG; ++j) {
-            const int it = i - LAG + j;
-            if (it >= 0) carry_apply(it, tq[j], eq[j]);
         }
     }
 

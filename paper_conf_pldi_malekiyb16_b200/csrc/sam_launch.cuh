@@ -124,13 +124,14 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     mcol<T>(geo.U, K, p.bu);
     constexpr int V = LB<T, K>::V;
     mcol<T>((int64_t)geo.Wn * V * geo.U, K, p.bwin);
+    mcol<T>((int64_t)geo.Wn * geo.U, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];
         mcol<T>((int64_t)v * Cfg<T>::ITEMS, K, b);
         for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
     }
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
-    for (int j = 0; j < MAX_LB; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
+    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
