@@ -52,13 +52,19 @@ template <typename T> struct Cfg;
 // ITEMS odd (bank-conflict-free strided smem reads); NB1 / NB2 smem buffers for local scans / carry
 // application + store; LAG = max tiles between local scan and carry application (the look-back's
 // latency budget, states in registers); PF = max claimed-but-unscanned tiles per CTA.
-template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
-template <> struct Cfg<float>    { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
-template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
-template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, LAG = 4, PF = 2; };
+template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, PF = 2; };
+template <> struct Cfg<float>    { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, PF = 2; };
+template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, PF = 2; };
+template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, PF = 2; };
+// Pending local states: small states (K * sizeof(T) <= 8 B per thread) wait in shared memory with
+// a deep ring (LAG = 12 tiles of slack for the look-back); larger ones in registers (LAG = 4).
+template <typename T, int K> struct Lag {
+    static constexpr bool SMEM = K * (int)sizeof(T) <= 8;
+    static constexpr int LAG = SMEM ? 12 : 4;
+};
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int NCARRY = 3;                          // carry (look-back) warps, round-robin over tiles
+constexpr int NCARRY = 4;                          // carry (look-back) warps, round-robin over tiles
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
 constexpr int TILE_THREADS = MAX_CWARPS * 32;
@@ -245,8 +251,9 @@ struct Smem {
     static constexpr int ITEMS = Cfg<T>::ITEMS;
     static constexpr int NB1 = Cfg<T>::NB1;
     static constexpr int NB2 = Cfg<T>::NB2;
-    static constexpr int LAG = Cfg<T>::LAG;
+    static constexpr int LAG = Lag<T, K>::LAG;
     static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
+    static constexpr int ELAG = Lag<T, K>::SMEM ? LAG : 0;          // smem-resident pending states
     static constexpr int TMAX = TILE_THREADS * ITEMS;
     static constexpr int NBL = 32;                // look-back binomial rows
     static constexpr int BUFB = ((TMAX * (int)sizeof(T) + 32) + 127) / 128 * 128;
@@ -263,7 +270,8 @@ struct Smem {
     static constexpr int OFF_BT = OFF_LA + NQ * LA * (int)sizeof(T);     // [K][32]
     static constexpr int OFF_BL = OFF_BT + K * 32 * (int)sizeof(T);      // [NBL][K]
     static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
-    static constexpr int BYTES = OFF_BQ + 8 * K * (int)sizeof(T);
+    static constexpr int OFF_EQ = OFF_BQ + 8 * K * (int)sizeof(T);       // [ELAG][TILE_THREADS][K]
+    static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
 };
 
 // ------------------------------------------------------------------------------------------
@@ -277,13 +285,15 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int NB1 = S::NB1;
     constexpr int NB2 = S::NB2;
     constexpr int NQ = S::NQ;
-    constexpr int LAG = Cfg<T>::LAG;
+    constexpr int LAG = S::LAG;
+    constexpr bool ESMEM = Lag<T, K>::SMEM;
     constexpr int PF = Cfg<T>::PF;
     constexpr int W2 = 2 * TagW<T>::W;  // tagged words per slot (aggregate + inclusive)
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
     static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 3, "ring sizes");
+    static_assert(S::BYTES <= 227 * 1024, "shared memory budget");
 
     extern __shared__ __align__(128) unsigned char smem[];
     uint64_t* bar_full1 = (uint64_t*)(smem + S::OFF_BAR);
@@ -821,7 +831,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // carry application (P2) runs once the producer has re-fetched it (its carry is known).
         // Up to LAG tiles may sit between P1 and P2; their local exclusive states wait in
         // registers (eq, a static ring indexed by iteration mod LAG).
-        T eq[LAG][K];
+        T eq[ESMEM ? 1 : LAG][K];
+        T* const eq_s = (T*)(smem + S::OFF_EQ);  // [LAG][TILE_THREADS][K] when ESMEM
         int p1_next = 0, p2_next = 0;
         for (;;) {
             const int end = *sm_end;
@@ -886,11 +897,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
                     }
                     mbar_arrive(&bar_p1[qs]);  // warp states ready; P1 buffer free for the producer
+                    if constexpr (ESMEM) {
 #pragma unroll
-                    for (int j = 0; j < LAG; ++j) {
-                        if (j == i % LAG) {
+                        for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + tid) * K + t] = e[t];
+                    } else {
 #pragma unroll
-                            for (int t = 0; t < K; ++t) eq[j][t] = e[t];
+                        for (int j = 0; j < LAG; ++j) {
+                            if (j == i % LAG) {
+#pragma unroll
+                                for (int t = 0; t < K; ++t) eq[j][t] = e[t];
+                            }
                         }
                     }
                     ++p1_next;
@@ -906,11 +922,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 if (ready) {
                     mbar_wait(&bar_full2[b2], par);
                     T e[K];
+                    if constexpr (ESMEM) {
 #pragma unroll
-                    for (int j = 0; j < LAG; ++j) {
-                        if (j == i % LAG) {
+                        for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + tid) * K + t];
+                    } else {
 #pragma unroll
-                            for (int t = 0; t < K; ++t) e[t] = eq[j][t];
+                        for (int j = 0; j < LAG; ++j) {
+                            if (j == i % LAG) {
+#pragma unroll
+                                for (int t = 0; t < K; ++t) e[t] = eq[j][t];
+                            }
                         }
                     }
                     carry_apply(i, tile_of[i % NQ], e);
