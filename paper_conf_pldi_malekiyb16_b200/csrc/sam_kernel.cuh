@@ -129,6 +129,15 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n}" ::"r"(smem_u32(bar)) : "memory");
 }
+// non-blocking probe (mbarrier.test_wait never suspends the thread; for event loops)
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    return ok != 0;
+}
 __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
@@ -388,9 +397,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 bulk_commit();  // one group per stored iteration (possibly empty)
             };
             int j1 = 0, j2 = 0, j3 = 0, jend = -1;
+            unsigned long long next_claim = atomicAdd(p.tile_ctr, 1ull);
             for (;;) {
                 // (1) store the oldest iteration whose carry application is done
-                if (j3 < j2 && mbar_try_wait(&bar_stored2[j3 % NB2], (uint32_t)((j3 / NB2) & 1))) {
+                if (j3 < j2 && mbar_test(&bar_stored2[j3 % NB2], (uint32_t)((j3 / NB2) & 1))) {
                     if (p.trace) SAM_TRACE(7, tile_of[j3 % NQ]);
                     store_tile(tile_of[j3 % NQ], smem + S::OFF_BUF2 + (j3 % NB2) * S::BUFB);
                     ++j3;
@@ -398,7 +408,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
                 // (2) reload (from L2) the next tile whose carry is known, into a free carry buffer
                 if (j2 < j1 && j2 - j3 < NB2 &&
-                    mbar_try_wait(&bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
+                    mbar_test(&bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
                     // groups committed after the store that last used this buffer (iteration j2-NB2)
                     const int later = j3 - 1 - (j2 - NB2);
                     if (later <= 0) bulk_wait_read<0>();
@@ -409,11 +419,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     ++j2;
                     continue;
                 }
-                // (3) claim and load a new tile (buffer free, at most PF unscanned, slot free)
+                // (3) claim and load a new tile (buffer free, at most PF unscanned, slot free).  The
+                // claim's atomic was issued one step earlier, so its round trip is off this path.
                 if (jend < 0 && j3 > j1 - NQ &&
-                    (j1 < NB1 || mbar_try_wait(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
-                    (j1 < PF || mbar_try_wait(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
-                    const unsigned long long t = atomicAdd(p.tile_ctr, 1ull);
+                    (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
+                    (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
+                    const unsigned long long t = next_claim;
+                    next_claim = atomicAdd(p.tile_ctr, 1ull);
                     if (t >= p.num_tiles) {
                         jend = j1;
                         *sm_end = j1;
@@ -427,6 +439,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     continue;
                 }
                 if (jend >= 0 && j3 == jend) break;
+                __nanosleep(16);
             }
             bulk_wait_all0();
         }
@@ -841,7 +854,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int i = p1_next;
                 const int b1 = i % NB1;
                 const uint32_t par = (uint32_t)((i / NB1) & 1);
-                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_try_wait(&bar_full1[b1], par) : 0, 0);
+                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full1[b1], par) : 0, 0);
                 if (ready) {
                     mbar_wait(&bar_full1[b1], par);
                     const int qs = i % NQ;
@@ -918,7 +931,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int i = p2_next;
                 const int b2 = i % NB2;
                 const uint32_t par = (uint32_t)((i / NB2) & 1);
-                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_try_wait(&bar_full2[b2], par) : 0, 0);
+                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full2[b2], par) : 0, 0);
                 if (ready) {
                     mbar_wait(&bar_full2[b2], par);
                     T e[K];
@@ -941,6 +954,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             } else if (end >= 0 && p1_next >= end) {
                 break;
             }
+            __nanosleep(32);  // nothing ready: yield issue slots to the other warps
         }
     }
 
