@@ -61,6 +61,8 @@ template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB1 = 3, NB2
 template <typename T, int K> struct Lag {
     static constexpr bool SMEM = K * (int)sizeof(T) <= 8;
     static constexpr int LAG = SMEM ? 12 : 4;
+    // super-tile: MMAX consecutive tiles claimed together, combined locally, one look-back
+    static constexpr int MMAX = SMEM ? 8 : 2;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
@@ -87,6 +89,8 @@ struct Params {
     uint64_t n;          // elements in this stream
     uint64_t h;          // virtual index of in[0] (= lane phase, 0 <= h < s)
     uint64_t num_tiles;  // ceil((h + n) / T)
+    uint64_t num_super;  // ceil(num_tiles / M)
+    int M;               // tiles per super-tile (look-back unit), 1..MMAX
     uint32_t delta;      // byte offset of virtual element 0 inside its 16-B chunk
     int s, G, logG, sp, c, logc, Pw, W, Wn;
     int U, T_, Uw;
@@ -102,12 +106,14 @@ struct Params {
     unsigned long long* trace;  // optional per-tile event timestamps [tile][8] (diagnostics), or null
     T bc[K];              // b_d(ITEMS)
     T bw[K];              // b_d(Uw)
-    T bu[K];              // b_d(U)
-    T bwin[K];            // b_d(Wn*V*U)   (one look-back round trip further)
-    T bwn[K];             // b_d(Wn*U)     (one window row further)
+    T bu[K];              // b_d(U)        (one tile)
+    T bus[K];             // b_d(M*U)      (one super-tile)
+    T bwin[K];            // b_d(Wn*V*M*U) (one look-back round trip further)
+    T bwn[K];             // b_d(Wn*M*U)   (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bq[8][K];           // b_d(q*Uw),     q < c
-    T bl[32][K];          // b_d(j*U),      j < Wn
+    T bl[32][K];          // b_d(j*M*U),    j < Wn
+    T bsub[8][K];         // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
 };
 
 // ------------------------------------------------------------------------------------------
@@ -273,10 +279,13 @@ struct Smem {
     static constexpr int OFF_BAR = OFF_BUF2 + NB2 * BUFB;  // full1[NB1] full2[NB2] stored2[NB2] p1/agg/carry[NQ]
     static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ;
     static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
-    static constexpr int OFF_TAG = OFF_TILE + NQ * 8;                    // u32 tag, i32 end iteration
-    static constexpr int OFF_WQ = (OFF_TAG + 8 + 15) / 16 * 16;          // NQ x [64][K]
+    static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
+    static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
+    static constexpr int OFF_TAG = OFF_SUB + NQ * 8;                     // u32 tag, i32 end, i32 agg progress
+    static constexpr int OFF_WQ = (OFF_TAG + 12 + 15) / 16 * 16;         // NQ x [64][K]
     static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
-    static constexpr int OFF_BT = OFF_LA + NQ * LA * (int)sizeof(T);     // [K][32]
+    static constexpr int OFF_LP = OFF_LA + NQ * LA * (int)sizeof(T);     // NQ x [8][K] in-super prefix
+    static constexpr int OFF_BT = OFF_LP + NQ * LA * (int)sizeof(T);     // [K][32]
     static constexpr int OFF_BL = OFF_BT + K * 32 * (int)sizeof(T);      // [NBL][K]
     static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
     static constexpr int OFF_EQ = OFF_BQ + 8 * K * (int)sizeof(T);       // [ELAG][TILE_THREADS][K]
@@ -312,8 +321,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint64_t* bar_agg = bar_p1 + NQ;
     uint64_t* bar_carry = bar_agg + NQ;
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
+    int64_t* sup_of = (int64_t*)(smem + S::OFF_SUP);
+    int* sub_of = (int*)(smem + S::OFF_SUB);  // [q][0] sub index, [q][1] sub-tiles in the super-tile
+    T* lp_all = (T*)(smem + S::OFF_LP);
     uint32_t* sm_tag = (uint32_t*)(smem + S::OFF_TAG);
     volatile int* sm_end = (volatile int*)(smem + S::OFF_TAG + 4);
+    volatile int* agg_done = (volatile int*)(smem + S::OFF_TAG + 8);  // iterations aggregated
     T* wq_all = (T*)(smem + S::OFF_WQ);
     T* la_all = (T*)(smem + S::OFF_LA);
     T* bt_s = (T*)(smem + S::OFF_BT);
@@ -342,6 +355,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         fence_mbar_init();
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
         *sm_end = -1;
+        *agg_done = 0;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
@@ -398,6 +412,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             };
             int j1 = 0, j2 = 0, j3 = 0, jend = -1;
             unsigned long long next_claim = atomicAdd(p.tile_ctr, 1ull);
+            int64_t cur_sup = -1;
+            int cur_j = 0, cur_cnt = 0;
             for (;;) {
                 // (1) store the oldest iteration whose carry application is done
                 if (j3 < j2 && mbar_test(&bar_stored2[j3 % NB2], (uint32_t)((j3 / NB2) & 1))) {
@@ -424,16 +440,29 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 if (jend < 0 && j3 > j1 - NQ &&
                     (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
                     (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
-                    const unsigned long long t = next_claim;
-                    next_claim = atomicAdd(p.tile_ctr, 1ull);
-                    if (t >= p.num_tiles) {
+                    if (cur_j == cur_cnt) {  // start the next super-tile
+                        cur_sup = (int64_t)next_claim;
+                        next_claim = atomicAdd(p.tile_ctr, 1ull);
+                        cur_j = 0;
+                        cur_cnt = 0;
+                        if ((uint64_t)cur_sup < p.num_super) {
+                            const uint64_t rest = p.num_tiles - (uint64_t)cur_sup * p.M;
+                            cur_cnt = rest < (uint64_t)p.M ? (int)rest : p.M;
+                        }
+                    }
+                    if (cur_cnt == 0) {
                         jend = j1;
                         *sm_end = j1;
                     } else {
-                        tile_of[j1 % NQ] = (int64_t)t;
+                        const int64_t t = cur_sup * p.M + cur_j;
+                        const int qs = j1 % NQ;
+                        tile_of[qs] = t;
+                        sup_of[qs] = cur_sup;
+                        sub_of[2 * qs] = cur_j;
+                        sub_of[2 * qs + 1] = cur_cnt;
+                        ++cur_j;
                         SAM_TRACE(0, t);
-                        load_tile((int64_t)t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1],
-                                  pol_keep);
+                        load_tile(t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1], pol_keep);
                         ++j1;
                     }
                     continue;
@@ -445,15 +474,25 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         }
     } else if (warp == NW + 1) {
         // =========================== aggregator warp: block combine, aggregate publish ===========
+        // Per tile: combine the warp states (E = warp-exclusive prefixes, tile aggregate A_j); per
+        // super-tile: the running prefix P_j = A_0 (+) ... (+) A_{j-1} (kept in registers by the
+        // lane that owns lane m's aggregate), and after the last sub-tile the super-tile aggregate,
+        // published for the other CTAs' look-backs (a4).
         const int npair = s * c;
+        T Pref[2][K];
         for (int i = 0;; ++i) {
             const int qs = i % NQ;
             if (!wait_or_end(&bar_p1[qs], (uint32_t)((i / NQ) & 1), i)) break;
             const int64_t tile = tile_of[qs];
+            const int64_t sup = sup_of[qs];
+            const int jsub = sub_of[2 * qs], cnt = sub_of[2 * qs + 1];
             if (lane == 0) SAM_TRACE(2, tile);
             T* wq = wq_all + qs * S::WQ;
             T* la = la_all + qs * S::LA;
-            for (int pair = lane; pair < 64; pair += 32) {
+            T* lp = lp_all + qs * S::LA;
+#pragma unroll
+            for (int ch = 0; ch < 2; ++ch) {
+                const int pair = lane + 32 * ch;
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
                 T E[K], yl[K];
@@ -479,12 +518,27 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 if (ok) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = E[t];  // warp-exclusive prefix
-                    if (qq == c - 1) {
+                    if (qq == c - 1) {  // this lane owns lane mm's tile aggregate yl
+                        if (jsub == 0) {
 #pragma unroll
-                        for (int t = 0; t < K; ++t) {
-                            la[mm * K + t] = yl[t];
-                            if (tile > 0) {  // a4: publish the tile aggregate
-                                put_tagged<T>(p.carry + (((size_t)tile * s + mm) * K + t) * W2, 0, tag, yl[t]);
+                            for (int t = 0; t < K; ++t) Pref[ch][t] = T(0);
+                        }
+#pragma unroll
+                        for (int t = 0; t < K; ++t) lp[mm * K + t] = Pref[ch][t];  // state before sub-tile
+#pragma unroll
+                        for (int t = K - 1; t >= 0; --t) {  // Pref <- M(U) Pref + A_j
+                            T acc2 = Pref[ch][t] + yl[t];
+#pragma unroll
+                            for (int j = 0; j < t; ++j) acc2 += p.bu[t - j] * Pref[ch][j];
+                            Pref[ch][t] = acc2;
+                        }
+                        if (jsub == cnt - 1) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) {
+                                la[mm * K + t] = Pref[ch][t];  // super-tile aggregate
+                                if (sup > 0) {  // a4: publish it
+                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W2, 0, tag, Pref[ch][t]);
+                                }
                             }
                         }
                     }
@@ -493,17 +547,34 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             __syncwarp();
             if (lane == 0) SAM_TRACE(3, tile);
             mbar_arrive(&bar_agg[qs]);
+            __syncwarp();
+            if (lane == 0) *agg_done = i + 1;
         }
     } else if (warp >= NW + 2) {
         // =========================== carry warps: decoupled look-back, inclusive states ==========
         const int npair = s * c;
-        for (int i = warp - (NW + 2);; i += NCARRY) {
-            const int qs = i % NQ;
-            if (!wait_or_end(&bar_agg[qs], (uint32_t)((i / NQ) & 1), i)) break;
-            const int64_t tile = tile_of[qs];
-            if (lane == 0) SAM_TRACE(4, tile);
-            T* wq = wq_all + qs * S::WQ;
-            const T* la = la_all + qs * S::LA;
+        for (int r = warp - (NW + 2);; r += NCARRY) {  // this CTA's r-th super-tile
+            const int i0 = r * p.M;                      // its first iteration
+            // Wait on the aggregator's progress counter first: a carry warp may run several
+            // super-tiles ahead of the aggregator, farther than the mbarrier parity can tell.
+            bool ended = false;
+            for (;;) {
+                if (*agg_done > i0) break;
+                const int end = *sm_end;
+                if (end >= 0 && i0 >= end) { ended = true; break; }
+                __nanosleep(64);
+            }
+            if (__any_sync(0xffffffffu, ended)) break;
+            mbar_wait(&bar_agg[i0 % NQ], (uint32_t)((i0 / NQ) & 1));  // acquire the slot data
+            const int cnt = sub_of[2 * (i0 % NQ) + 1];
+            const int il = i0 + cnt - 1;                 // its last iteration
+            if (cnt > 1) {
+                while (*agg_done <= il) __nanosleep(64);
+                mbar_wait(&bar_agg[il % NQ], (uint32_t)((il / NQ) & 1));
+            }
+            const int64_t tile = sup_of[i0 % NQ];        // look-back unit: the super-tile
+            if (lane == 0) SAM_TRACE(4, tile_of[i0 % NQ]);
+            const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
 
@@ -684,37 +755,53 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 for (int t = 0; t < K; ++t) C[t] = total[t];
             }
 
-            // publish the inclusive state of this tile: M(U) C + A
-            if ((uint64_t)tile + 1 < p.num_tiles && lane_ok) {
+            // publish the inclusive state of this super-tile: M(M U) C + A
+            if ((uint64_t)tile + 1 < p.num_super && lane_ok) {
                 unsigned long long* const carry_tile = p.carry + (size_t)tile * s * K * W2;
 #pragma unroll
                 for (int t = 0; t < K; ++t) {
                     T acc2 = C[t] + la[ml * K + t];
 #pragma unroll
-                    for (int j = 0; j < t; ++j) acc2 += p.bu[t - j] * C[j];
+                    for (int j = 0; j < t; ++j) acc2 += p.bus[t - j] * C[j];
                     put_tagged<T>(carry_tile + (lane * K + t) * W2, 1, tag, acc2);
                 }
             }
-            // per-warp incoming states C_{m,q} = M(q*Uw) C_m + E_{m,q}  (E in wq, from the combine)
-            for (int pair = lane; pair < 64; pair += 32) {
-                const bool ok = pair < npair;
-                const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
-                T Cm[K];
+            // each sub-tile j: C_j = M(j U) C + P_j, then per-warp incoming states
+            // C_{m,q} = M(q*Uw) C_{j,m} + E_{m,q}  (E in wq, from the combine)
+            for (int j = 0; j < cnt; ++j) {
+                const int qj = (i0 + j) % NQ;
+                T* wq = wq_all + qj * S::WQ;
+                const T* lp = lp_all + qj * S::LA;
+                T Cj[K];
 #pragma unroll
-                for (int t = 0; t < K; ++t) Cm[t] = shfl_idx(C[t], mm);
-                if (ok) {
+                for (int t = K - 1; t >= 0; --t) {
+                    T acc2 = C[t] + lp[ml * K + t];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) {
-                        T acc2 = Cm[t] + wq[(qq * s + mm) * K + t];
+                    for (int d = 0; d < t; ++d) acc2 += p.bsub[j][t - d] * C[d];
+                    Cj[t] = acc2;
+                }
 #pragma unroll
-                        for (int j = 0; j < t; ++j) acc2 += bq_s[qq * K + (t - j)] * Cm[j];
-                        wq[(qq * s + mm) * K + t] = acc2;
+                for (int ch = 0; ch < 2; ++ch) {
+                    const int pair = lane + 32 * ch;
+                    const bool ok = pair < npair;
+                    const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
+                    T Cm[K];
+#pragma unroll
+                    for (int t = 0; t < K; ++t) Cm[t] = shfl_idx(Cj[t], mm);
+                    if (ok) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) {
+                            T acc2 = Cm[t] + wq[(qq * s + mm) * K + t];
+#pragma unroll
+                            for (int d = 0; d < t; ++d) acc2 += bq_s[qq * K + (t - d)] * Cm[d];
+                            wq[(qq * s + mm) * K + t] = acc2;
+                        }
                     }
                 }
+                __syncwarp();
+                if (lane == 0) SAM_TRACE(5, tile_of[qj]);
+                mbar_arrive(&bar_carry[qj]);
             }
-            __syncwarp();
-            if (lane == 0) SAM_TRACE(5, tile);
-            mbar_arrive(&bar_carry[qs]);
         }
     } else {
         // =========================== compute warps ===============================================

@@ -119,19 +119,30 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     p.done_ctr = a.done_ctr;
     p.epoch_ptr = a.epoch_ptr;
     p.trace = a.trace;
+    // super-tile size: up to MMAX tiles per look-back unit, but keep >= 2 super-tiles per SM
+    {
+        uint64_t m = p.num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
+        if (m < 1) m = 1;
+        if (m > (uint64_t)Lag<T, K>::MMAX) m = Lag<T, K>::MMAX;
+        p.M = (int)m;
+        p.num_super = (p.num_tiles + m - 1) / m;
+    }
+    const int64_t US = (int64_t)p.M * geo.U;  // lane length of a super-tile
     mcol<T>(Cfg<T>::ITEMS, K, p.bc);
     mcol<T>(geo.Uw, K, p.bw);
     mcol<T>(geo.U, K, p.bu);
+    mcol<T>(US, K, p.bus);
     constexpr int V = LB<T, K>::V;
-    mcol<T>((int64_t)geo.Wn * V * geo.U, K, p.bwin);
-    mcol<T>((int64_t)geo.Wn * geo.U, K, p.bwn);
+    mcol<T>((int64_t)geo.Wn * V * US, K, p.bwin);
+    mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];
         mcol<T>((int64_t)v * Cfg<T>::ITEMS, K, b);
         for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
     }
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
-    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * geo.U, K, p.bl[j]);
+    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, p.bl[j]);
+    for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, p.bsub[j]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
