@@ -52,17 +52,22 @@ template <typename T> struct Cfg;
 // ITEMS odd (bank-conflict-free strided smem reads); NB1 / NB2 smem buffers for local scans / carry
 // application + store; LAG = max tiles between local scan and carry application (the look-back's
 // latency budget, states in registers); PF = max claimed-but-unscanned tiles per CTA.
-template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, PF = 2; };
-template <> struct Cfg<float>    { static constexpr int ITEMS = 31, NB1 = 3, NB2 = 3, PF = 2; };
-template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, PF = 2; };
-template <> struct Cfg<double>   { static constexpr int ITEMS = 15, NB1 = 3, NB2 = 3, PF = 2; };
-// Pending local states: small states (K * sizeof(T) <= 8 B per thread) wait in shared memory with
-// a deep ring (LAG = 12 tiles of slack for the look-back); larger ones in registers (LAG = 4).
+template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31; };
+template <> struct Cfg<float>    { static constexpr int ITEMS = 31; };
+template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15; };
+template <> struct Cfg<double>   { static constexpr int ITEMS = 15; };
+// Pipeline shape by per-thread state size K * sizeof(T):
+//   <= 8 B : 4 local-scan buffers, 2 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
+//   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
+//   larger : 3 + 2 buffers, pending states in registers (LAG = 4), super-tiles of 2
 template <typename T, int K> struct Lag {
-    static constexpr bool SMEM = K * (int)sizeof(T) <= 8;
-    static constexpr int LAG = SMEM ? 12 : 4;
-    // super-tile: MMAX consecutive tiles claimed together, combined locally, one look-back
-    static constexpr int MMAX = SMEM ? 8 : 2;
+    static constexpr int SB = K * (int)sizeof(T);
+    static constexpr bool SMEM = SB <= 16;           // pending local states in shared memory
+    static constexpr int LAG = SB <= 8 ? 12 : (SB <= 16 ? 8 : 4);
+    static constexpr int MMAX = SB <= 8 ? 4 : 2;     // max tiles per super-tile (look-back unit)
+    static constexpr int NB1 = SB <= 8 ? 4 : 3;      // local-scan (HBM) buffers
+    static constexpr int NB2 = 2;                    // carry-application (L2 reload) buffers
+    static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
@@ -264,8 +269,8 @@ template <> struct IsInt<uint64_t> { static constexpr bool value = true; };
 template <typename T, int K>
 struct Smem {
     static constexpr int ITEMS = Cfg<T>::ITEMS;
-    static constexpr int NB1 = Cfg<T>::NB1;
-    static constexpr int NB2 = Cfg<T>::NB2;
+    static constexpr int NB1 = Lag<T, K>::NB1;
+    static constexpr int NB2 = Lag<T, K>::NB2;
     static constexpr int LAG = Lag<T, K>::LAG;
     static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
     static constexpr int ELAG = Lag<T, K>::SMEM ? LAG : 0;          // smem-resident pending states
@@ -305,7 +310,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int NQ = S::NQ;
     constexpr int LAG = S::LAG;
     constexpr bool ESMEM = Lag<T, K>::SMEM;
-    constexpr int PF = Cfg<T>::PF;
+    constexpr int PF = Lag<T, K>::PF;
     constexpr int W2 = 2 * TagW<T>::W;  // tagged words per slot (aggregate + inclusive)
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
