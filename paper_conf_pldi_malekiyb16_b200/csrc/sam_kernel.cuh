@@ -57,7 +57,7 @@ template <> struct Cfg<float>    { static constexpr int ITEMS = 31; };
 template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15; };
 template <> struct Cfg<double>   { static constexpr int ITEMS = 15; };
 // Pipeline shape by per-thread state size K * sizeof(T):
-//   <= 8 B : 4 local-scan buffers, 2 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
+//   <= 8 B : 3 local-scan buffers, 3 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
 //   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
 //   larger : 3 + 2 buffers, pending states in registers (LAG = 4), super-tiles of 2
 template <typename T, int K> struct Lag {
@@ -65,8 +65,8 @@ template <typename T, int K> struct Lag {
     static constexpr bool SMEM = SB <= 16;           // pending local states in shared memory
     static constexpr int LAG = SB <= 8 ? 12 : (SB <= 16 ? 8 : 4);
     static constexpr int MMAX = SB <= 8 ? 4 : 2;     // max tiles per super-tile (look-back unit)
-    static constexpr int NB1 = SB <= 8 ? 4 : 3;      // local-scan (HBM) buffers
-    static constexpr int NB2 = 2;                    // carry-application (L2 reload) buffers
+    static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
+    static constexpr int NB2 = SB <= 8 ? 3 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
 };
 
