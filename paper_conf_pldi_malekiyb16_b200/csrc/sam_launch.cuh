@@ -3,6 +3,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <mutex>
@@ -124,6 +125,10 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
         uint64_t m = p.num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
         if (m < 1) m = 1;
         if (m > (uint64_t)Lag<T, K>::MMAX) m = Lag<T, K>::MMAX;
+        if (const char* env = getenv("SAM_SUPER_TILE")) {  // experiments: force a smaller super-tile
+            const int f = atoi(env);
+            if (f >= 1 && (uint64_t)f < m) m = (uint64_t)f;
+        }
         p.M = (int)m;
         p.num_super = (p.num_tiles + m - 1) / m;
     }
