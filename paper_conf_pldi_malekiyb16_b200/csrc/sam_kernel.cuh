@@ -68,12 +68,20 @@ template <typename T, int K> struct Lag {
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
     static constexpr int NB2 = SB <= 8 ? 3 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
+    // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
+    // carry applications (P2) (measured faster there; order 1 keeps one group)
+    static constexpr bool SPLIT = SMEM && K >= 2;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
 constexpr int NCARRY = 4;                          // carry (look-back) warps, round-robin over tiles
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
+// threads of a CTA: one compute group (or two: local scans + carry applications) + service warps
+template <typename T, int K> struct Threads {
+    static constexpr int GROUPS = Lag<T, K>::SPLIT ? 2 : 1;
+    static constexpr int VALUE = (GROUPS * MAX_CWARPS + SERVICE_WARPS) * 32;
+};
 constexpr int TILE_THREADS = MAX_CWARPS * 32;
 
 enum StoreMode { STORE_BULK = 0, STORE_STRIPED = 1, STORE_NONE = 2 };
@@ -287,7 +295,7 @@ struct Smem {
     static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
     static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
     static constexpr int OFF_TAG = OFF_SUB + NQ * 8;                     // u32 tag, i32 end, i32 agg progress
-    static constexpr int OFF_WQ = (OFF_TAG + 12 + 15) / 16 * 16;         // NQ x [64][K]
+    static constexpr int OFF_WQ = (OFF_TAG + 16 + 15) / 16 * 16;         // NQ x [64][K]
     static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
     static constexpr int OFF_LP = OFF_LA + NQ * LA * (int)sizeof(T);     // NQ x [8][K] in-super prefix
     static constexpr int OFF_BT = OFF_LP + NQ * LA * (int)sizeof(T);     // [K][32]
@@ -301,7 +309,7 @@ struct Smem {
 // the kernel
 // ------------------------------------------------------------------------------------------
 template <typename T, int K>
-__global__ void __launch_bounds__(MAX_THREADS, 1)
+__global__ void __launch_bounds__(Threads<T, K>::VALUE, 1)
 sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     using S = Smem<T, K>;
     constexpr int ITEMS = S::ITEMS;
@@ -341,8 +349,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
     const int s = p.s, c = p.c;
-    const int NW = p.W;          // compute warps
-    const int NCT = NW * 32;     // compute threads
+    constexpr bool SPLIT = Lag<T, K>::SPLIT;
+    const int NW = p.W;          // compute warps per group
+    const int NCT = NW * 32;     // compute threads per group
+    const int NCW = SPLIT ? 2 * NW : NW;  // compute warps (both groups); service warps follow
     const int Tt = p.T_;
 
     // ---- prologue: barriers, tables, epoch tag -------------------------------------------------
@@ -361,6 +371,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
         *sm_end = -1;
         *agg_done = 0;
+        *(volatile int*)(smem + S::OFF_TAG + 12) = 0;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
@@ -378,7 +389,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         return !__any_sync(0xffffffffu, ended);
     };
 
-    if (warp == NW) {
+    if (warp == NCW) {
         // =========================== producer warp: claims, loads, reloads, stores =============
         if (lane == 0) {
             const uint64_t pol_keep = policy_evict_last();
@@ -477,7 +488,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             }
             bulk_wait_all0();
         }
-    } else if (warp == NW + 1) {
+    } else if (warp == NCW + 1) {
         // =========================== aggregator warp: block combine, aggregate publish ===========
         // Per tile: combine the warp states (E = warp-exclusive prefixes, tile aggregate A_j); per
         // super-tile: the running prefix P_j = A_0 (+) ... (+) A_{j-1} (kept in registers by the
@@ -555,10 +566,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             __syncwarp();
             if (lane == 0) *agg_done = i + 1;
         }
-    } else if (warp >= NW + 2) {
+    } else if (warp >= NCW + 2) {
         // =========================== carry warps: decoupled look-back, inclusive states ==========
         const int npair = s * c;
-        for (int r = warp - (NW + 2);; r += NCARRY) {  // this CTA's r-th super-tile
+        for (int r = warp - (NCW + 2);; r += NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;                      // its first iteration
             // Wait on the aggregator's progress counter first: a carry warp may run several
             // super-tiles ahead of the aggregator, farther than the mbarrier parity can tell.
@@ -810,8 +821,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         }
     } else {
         // =========================== compute warps ===============================================
+        const bool is_p2_group = SPLIT && warp >= NW;  // SPLIT: warps [NW, 2NW) apply carries
+        const int cwarp = warp % NW;                   // warp within its group
+        const int gtid = tid % NCT;                    // thread within its group
         const int G = p.G, Pw = p.Pw;
-        const int g = warp % p.sp, q = warp / p.sp;
+        const int g = cwarp % p.sp, q = cwarp / p.sp;
         const int a = lane & (G - 1), v = lane >> p.logG;
         const int m = g * G + a;
         const int u = q * Pw + v;
@@ -821,7 +835,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         auto carry_apply = [&](int it, int64_t tile, const T* e) {
             const int b2 = it % NB2;
             const int qs = it % NQ;
-            if (tid == 0) SAM_TRACE(6, tile);
+            if (gtid == 0) SAM_TRACE(6, tile);
             T* xs = (T*)(smem + S::OFF_BUF2 + b2 * S::BUFB + p.delta);
             const T* wq = wq_all + qs * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
@@ -925,128 +939,159 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if (p.store_mode == STORE_BULK) {
                 fence_proxy_async_smem();
             } else if (p.store_mode == STORE_STRIPED) {
-                named_bar_sync(2, NCT);
-                for (uint64_t ve = lo + tid; ve < hi; ve += NCT) p.out[ve - p.h] = xs[ve - e0];
+                named_bar_sync(2 + (is_p2_group ? 1 : 0), NCT);
+                for (uint64_t ve = lo + gtid; ve < hi; ve += NCT) p.out[ve - p.h] = xs[ve - e0];
             }
             mbar_arrive(&bar_stored2[b2]);
         };
 
-        // Scheduling: a loaded tile's local scan (P1) always goes first, so its aggregate is
-        // published as early as possible (predecessor aggregates gate every look-back); a tile's
-        // carry application (P2) runs once the producer has re-fetched it (its carry is known).
-        // Up to LAG tiles may sit between P1 and P2; their local exclusive states wait in
-        // registers (eq, a static ring indexed by iteration mod LAG).
-        T eq[ESMEM ? 1 : LAG][K];
-        T* const eq_s = (T*)(smem + S::OFF_EQ);  // [LAG][TILE_THREADS][K] when ESMEM
-        int p1_next = 0, p2_next = 0;
-        for (;;) {
-            const int end = *sm_end;
-            // ---- P1 of the next loaded tile, if the state ring has room ---------------------------
-            if ((end < 0 || p1_next < end) && p1_next < p2_next + LAG) {
-                const int i = p1_next;
-                const int b1 = i % NB1;
-                const uint32_t par = (uint32_t)((i / NB1) & 1);
-                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full1[b1], par) : 0, 0);
-                if (ready) {
-                    mbar_wait(&bar_full1[b1], par);
-                    const int qs = i % NQ;
-                    const int64_t tile = tile_of[qs];
-                    if (tid == 0) SAM_TRACE(1, tile);
-                    const T* xs = (const T*)(smem + S::OFF_BUF1 + b1 * S::BUFB + p.delta);
-                    T* wq = wq_all + qs * S::WQ;
-                    const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
-                    const bool masked = (e0 < p.h) || (e0 + Tt > p.h + p.n);
-                    // a2/a3: lane run, thread-serial zero-seeded recurrence
-                    T acc[K];
+        // a3 for iteration i (tile loaded in local-scan buffer b1): zero-seeded local scan, warp
+        // states to wq, returns the thread's local exclusive state e
+        auto local_scan = [&](int i, int b1, T* e) {
+            const int qs = i % NQ;
+            const int64_t tile = tile_of[qs];
+            if (gtid == 0) SAM_TRACE(1, tile);
+            const T* xs = (const T*)(smem + S::OFF_BUF1 + b1 * S::BUFB + p.delta);
+            T* wq = wq_all + qs * S::WQ;
+            const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
+            const bool masked = (e0 < p.h) || (e0 + Tt > p.h + p.n);
+            // a2/a3: lane run, thread-serial zero-seeded recurrence
+            T acc[K];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) acc[t] = T(0);
-                    if (!masked) {
+            for (int t = 0; t < K; ++t) acc[t] = T(0);
+            if (!masked) {
 #pragma unroll
-                        for (int it = 0; it < ITEMS; ++it) {
-                            const T x = xs[base_loc + it * s];
-                            acc[0] += x;
+                for (int it = 0; it < ITEMS; ++it) {
+                    const T x = xs[base_loc + it * s];
+                    acc[0] += x;
 #pragma unroll
-                            for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
-                        }
-                    } else {
+                    for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                }
+            } else {
 #pragma unroll
-                        for (int it = 0; it < ITEMS; ++it) {
-                            const int el = base_loc + it * s;
-                            const uint64_t ve = e0 + el;
-                            const T x = (ve >= p.h && ve < p.h + p.n) ? xs[el] : T(0);
-                            acc[0] += x;
+                for (int it = 0; it < ITEMS; ++it) {
+                    const int el = base_loc + it * s;
+                    const uint64_t ve = e0 + el;
+                    const T x = (ve >= p.h && ve < p.h + p.n) ? xs[el] : T(0);
+                    acc[0] += x;
 #pragma unroll
-                            for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
-                        }
-                    }
-                    // a3: warp scan of thread states (order by order, plain shuffle scans)
-                    // e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
-                    // z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]
-                    T e[K];
-#pragma unroll
-                    for (int t = 0; t < K; ++t) {
-                        T z = acc[t];
-#pragma unroll
-                        for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
-                        T y = z;
-                        for (int off = G; off < 32; off <<= 1) {
-                            T o = shfl_up(y, off);
-                            if (lane >= off) y += o;
-                        }
-                        if constexpr (IsInt<T>::value) {
-                            e[t] = y - z;
-                        } else {
-                            T o = shfl_up(y, G);
-                            e[t] = (lane >= G) ? o : T(0);
-                        }
-                        if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
-                    }
-                    mbar_arrive(&bar_p1[qs]);  // warp states ready; P1 buffer free for the producer
-                    if constexpr (ESMEM) {
-#pragma unroll
-                        for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + tid) * K + t] = e[t];
-                    } else {
-#pragma unroll
-                        for (int j = 0; j < LAG; ++j) {
-                            if (j == i % LAG) {
-#pragma unroll
-                                for (int t = 0; t < K; ++t) eq[j][t] = e[t];
-                            }
-                        }
-                    }
-                    ++p1_next;
-                    continue;
+                    for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
                 }
             }
-            // ---- P2 of the oldest scanned tile once it has been re-fetched with its carry --------
-            if (p2_next < p1_next) {
-                const int i = p2_next;
-                const int b2 = i % NB2;
-                const uint32_t par = (uint32_t)((i / NB2) & 1);
-                const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full2[b2], par) : 0, 0);
-                if (ready) {
-                    mbar_wait(&bar_full2[b2], par);
+            // a3: warp scan of thread states (order by order, plain shuffle scans)
+            // e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
+            // z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]
+#pragma unroll
+            for (int t = 0; t < K; ++t) {
+                T z = acc[t];
+#pragma unroll
+                for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
+                T y = z;
+                for (int off = G; off < 32; off <<= 1) {
+                    T o = shfl_up(y, off);
+                    if (lane >= off) y += o;
+                }
+                if constexpr (IsInt<T>::value) {
+                    e[t] = y - z;
+                } else {
+                    T o = shfl_up(y, G);
+                    e[t] = (lane >= G) ? o : T(0);
+                }
+                if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
+            }
+            mbar_arrive(&bar_p1[qs]);  // warp states ready; P1 buffer free for the producer
+        };
+
+        T* const eq_s = (T*)(smem + S::OFF_EQ);  // [LAG][TILE_THREADS][K] pending states (ESMEM)
+        volatile int* p2_cnt = (volatile int*)(smem + S::OFF_TAG + 12);  // SPLIT: P2 warp-tiles done
+        if constexpr (SPLIT) {
+            // Two groups: local scans never wait behind carry applications and vice versa.
+            if (!is_p2_group) {
+                for (int i = 0;; ++i) {
+                    const int b1 = i % NB1;
+                    if (!wait_or_end(&bar_full1[b1], (uint32_t)((i / NB1) & 1), i)) break;
+                    // the pending-state slot i % LAG must have been consumed by P2 of i - LAG
+                    while (*p2_cnt < (i - LAG + 1) * NW) __nanosleep(32);
                     T e[K];
-                    if constexpr (ESMEM) {
+                    local_scan(i, b1, e);
 #pragma unroll
-                        for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + tid) * K + t];
-                    } else {
+                    for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                }
+            } else {
+                for (int i = 0;; ++i) {
+                    const int b2 = i % NB2;
+                    if (!wait_or_end(&bar_full2[b2], (uint32_t)((i / NB2) & 1), i)) break;
+                    T e[K];
 #pragma unroll
-                        for (int j = 0; j < LAG; ++j) {
-                            if (j == i % LAG) {
-#pragma unroll
-                                for (int t = 0; t < K; ++t) e[t] = eq[j][t];
-                            }
-                        }
-                    }
+                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
                     carry_apply(i, tile_of[i % NQ], e);
-                    ++p2_next;
-                    continue;
+                    __syncwarp();
+                    if (lane == 0) atomicAdd((int*)p2_cnt, 1);
                 }
-            } else if (end >= 0 && p1_next >= end) {
-                break;
             }
-            __nanosleep(32);  // nothing ready: yield issue slots to the other warps
+        } else {
+            // One group.  A loaded tile's local scan (P1) always goes first, so its aggregate is
+            // published as early as possible (predecessor aggregates gate every look-back); a
+            // tile's carry application (P2) runs once the producer has re-fetched it.  Up to LAG
+            // tiles sit between P1 and P2, their local states in registers (static ring eq).
+            T eq[ESMEM ? 1 : LAG][K];  // register ring only when the states do not fit smem
+            int p1_next = 0, p2_next = 0;
+            for (;;) {
+                const int end = *sm_end;
+                if ((end < 0 || p1_next < end) && p1_next < p2_next + LAG) {
+                    const int i = p1_next;
+                    const int b1 = i % NB1;
+                    const uint32_t par = (uint32_t)((i / NB1) & 1);
+                    const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full1[b1], par) : 0, 0);
+                    if (ready) {
+                        mbar_wait(&bar_full1[b1], par);
+                        T e[K];
+                        local_scan(i, b1, e);
+                        if constexpr (ESMEM) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                        } else {
+#pragma unroll
+                            for (int j = 0; j < LAG; ++j) {
+                                if (j == i % LAG) {
+#pragma unroll
+                                    for (int t = 0; t < K; ++t) eq[j][t] = e[t];
+                                }
+                            }
+                        }
+                        ++p1_next;
+                        continue;
+                    }
+                }
+                if (p2_next < p1_next) {
+                    const int i = p2_next;
+                    const int b2 = i % NB2;
+                    const uint32_t par = (uint32_t)((i / NB2) & 1);
+                    const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full2[b2], par) : 0, 0);
+                    if (ready) {
+                        mbar_wait(&bar_full2[b2], par);
+                        T e[K];
+                        if constexpr (ESMEM) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
+                        } else {
+#pragma unroll
+                            for (int j = 0; j < LAG; ++j) {
+                                if (j == i % LAG) {
+#pragma unroll
+                                    for (int t = 0; t < K; ++t) e[t] = eq[j][t];
+                                }
+                            }
+                        }
+                        carry_apply(i, tile_of[i % NQ], e);
+                        ++p2_next;
+                        continue;
+                    }
+                } else if (end >= 0 && p1_next >= end) {
+                    break;
+                }
+                __nanosleep(32);  // nothing ready: yield issue slots to the other warps
+            }
         }
     }
 

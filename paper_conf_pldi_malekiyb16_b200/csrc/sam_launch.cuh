@@ -86,7 +86,7 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES);
             if (e != cudaSuccess) return e;
             int nb = 0;
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K>, MAX_THREADS, S::BYTES);
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K>, Threads<T, K>::VALUE, S::BYTES);
             if (e != cudaSuccess) return e;
             info.max_blocks_per_sm = nb > 0 ? nb : 1;
             info.ready = true;
@@ -153,7 +153,7 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
     if (grid > p.num_tiles) grid = p.num_tiles;
     if (grid < 1) grid = 1;
-    sam_scan_kernel<T, K><<<(unsigned)grid, (geo.W + SERVICE_WARPS) * 32, S::BYTES, a.stream>>>(p);
+    sam_scan_kernel<T, K><<<(unsigned)grid, (Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32, S::BYTES, a.stream>>>(p);
     if (launches) ++*launches;
     return cudaGetLastError();
 }
