@@ -4,6 +4,7 @@
 // of sam_kernel.cuh; this file only validates, allocates and launches.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <atomic>
@@ -71,12 +72,26 @@ std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
 std::map<int, int> g_sms;
 unsigned long long* g_trace = nullptr;  // diagnostics: per-tile event timestamps of the next launches
 
+// First use of a device: SM count, and an L2 persisting set-aside so the kernel's L2::evict_last
+// hints (tiles parked in L2 between local scan and carry application) are honoured.  Only raised,
+// never lowered; SAM_L2_PERSIST_MB=0 disables it.
 int num_sms(int dev) {
     auto it = g_sms.find(dev);
     if (it != g_sms.end()) return it->second;
     int n = 0;
     if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
     g_sms[dev] = n;
+    int maxp = 0;
+    size_t cur = 0;
+    long want_mb = 0;  // measured: a set-aside starves the streaming traffic; opt in only
+    if (const char* env = getenv("SAM_L2_PERSIST_MB")) want_mb = atol(env);
+    if (want_mb > 0 && cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) == cudaSuccess &&
+        maxp > 0 && cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess) {
+        size_t want = (size_t)want_mb << 20;
+        if (want > (size_t)maxp) want = (size_t)maxp;
+        if (cur < want) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+    }
+    cudaGetLastError();  // the set-aside is an optimisation; never fail a scan over it
     return n;
 }
 
