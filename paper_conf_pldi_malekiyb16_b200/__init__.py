@@ -171,3 +171,9 @@ def scan_host(x, order: int = 1, tuple: int = 1, inclusive: bool = True, out=Non
     sam_scan_host(dtype_code(x.dtype), order, tuple, inclusive, ctypes.c_void_p(x.data_ptr()),
                   ctypes.c_void_p(out.data_ptr()), x.numel(), _stream_ptr(stream))
     return out
+
+
+def tile_items(dtype_name: str) -> int:
+    """Items per thread of the kernel's tile geometry (mirrors sam::Cfg<T>::ITEMS; tests use it to
+    place sizes at tile boundaries)."""
+    return {"i32": 27, "f32": 27, "i64": 13, "f64": 13}[dtype_name]

@@ -52,10 +52,10 @@ template <typename T> struct Cfg;
 // ITEMS odd (bank-conflict-free strided smem reads); NB1 / NB2 smem buffers for local scans / carry
 // application + store; LAG = max tiles between local scan and carry application (the look-back's
 // latency budget, states in registers); PF = max claimed-but-unscanned tiles per CTA.
-template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 31; };
-template <> struct Cfg<float>    { static constexpr int ITEMS = 31; };
-template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 15; };
-template <> struct Cfg<double>   { static constexpr int ITEMS = 15; };
+template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 27; };
+template <> struct Cfg<float>    { static constexpr int ITEMS = 27; };
+template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 13; };
+template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
 // Pipeline shape by per-thread state size K * sizeof(T):
 //   <= 8 B : 3 local-scan buffers, 3 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
 //   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
@@ -66,7 +66,7 @@ template <typename T, int K> struct Lag {
     static constexpr int LAG = SB <= 8 ? 12 : (SB <= 16 ? 8 : 4);
     static constexpr int MMAX = SB <= 8 ? 4 : 2;     // max tiles per super-tile (look-back unit)
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
-    static constexpr int NB2 = SB <= 8 ? 3 : 2;      // carry-application (L2 reload) buffers
+    static constexpr int NB2 = SB <= 8 ? 4 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
@@ -323,7 +323,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
-    static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 3, "ring sizes");
+    static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 4, "ring sizes");
     static_assert(S::BYTES <= 227 * 1024, "shared memory budget");
 
     extern __shared__ __align__(128) unsigned char smem[];
@@ -445,7 +445,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     const int later = j3 - 1 - (j2 - NB2);
                     if (later <= 0) bulk_wait_read<0>();
                     else if (later == 1) bulk_wait_read<1>();
-                    else bulk_wait_read<2>();
+                    else if (later == 2) bulk_wait_read<2>();
+                    else bulk_wait_read<3>();
                     load_tile(tile_of[j2 % NQ], smem + S::OFF_BUF2 + (j2 % NB2) * S::BUFB, &bar_full2[j2 % NB2],
                               pol_stream);
                     ++j2;

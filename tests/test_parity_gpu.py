@@ -78,7 +78,8 @@ def tile_elems(s, items):
 
 @pytest.mark.parametrize("k,s", [(1, 1), (3, 2), (8, 8), (2, 5), (4, 3), (1, 7)])
 def test_edge_sizes(k, s):
-    for name, items in (("i32", 31), ("i64", 15)):
+    from paper_conf_pldi_malekiyb16_b200 import tile_items
+    for name, items in (("i32", tile_items("i32")), ("i64", tile_items("i64"))):
         T = tile_elems(s, items)
         for n in sorted({1, 2, 3, s - 1 if s > 1 else 1, s, s + 1, 31, 32, 33, T - 1, T, T + 1, 2 * T - 1,
                          2 * T + 3, 3 * T + 5, 7 * T + s}):
