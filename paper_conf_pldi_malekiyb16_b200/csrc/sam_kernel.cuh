@@ -290,12 +290,13 @@ struct Smem {
     static constexpr int OFF_BUF1 = 0;
     static constexpr int OFF_BUF2 = OFF_BUF1 + NB1 * BUFB;
     static constexpr int OFF_BAR = OFF_BUF2 + NB2 * BUFB;  // full1[NB1] full2[NB2] stored2[NB2] p1/agg/carry[NQ]
-    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ;
+    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ + NCARRY;
     static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
     static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
     static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
     static constexpr int OFF_TAG = OFF_SUB + NQ * 8;                     // u32 tag, i32 end, i32 agg progress
-    static constexpr int OFF_WQ = (OFF_TAG + 16 + 15) / 16 * 16;         // NQ x [64][K]
+    static constexpr int OFF_CW = OFF_TAG + 16;                          // NCARRY x i32 super-tile taken
+    static constexpr int OFF_WQ = (OFF_CW + 4 * NCARRY + 15) / 16 * 16;  // NQ x [64][K]
     static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
     static constexpr int OFF_LP = OFF_LA + NQ * LA * (int)sizeof(T);     // NQ x [8][K] in-super prefix
     static constexpr int OFF_BT = OFF_LP + NQ * LA * (int)sizeof(T);     // [K][32]
@@ -333,6 +334,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint64_t* bar_p1 = bar_stored2 + NB2;
     uint64_t* bar_agg = bar_p1 + NQ;
     uint64_t* bar_carry = bar_agg + NQ;
+    uint64_t* bar_cw = bar_carry + NQ;  // [NCARRY]: a super-tile is ready for carry warp w
+    volatile int* cw_taken = (volatile int*)(smem + S::OFF_CW);  // last super-tile each carry warp took
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
     int64_t* sup_of = (int64_t*)(smem + S::OFF_SUP);
     int* sub_of = (int*)(smem + S::OFF_SUB);  // [q][0] sub index, [q][1] sub-tiles in the super-tile
@@ -366,6 +369,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             mbar_init(&bar_p1[q], NCT);
             mbar_init(&bar_agg[q], 32);
             mbar_init(&bar_carry[q], 32);
+        }
+        for (int w = 0; w < NCARRY; ++w) {
+            mbar_init(&bar_cw[w], 32);
+            cw_taken[w] = -1;
         }
         fence_mbar_init();
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
@@ -519,9 +526,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                     for (int j = 0; j < t; ++j) z += p.bw[t - j] * E[j];
                     T y = z;
-                    for (int off = 1; off < c; off <<= 1) {
-                        T o = shfl_up(y, off);
-                        if (qq >= off) y += o;
+#pragma unroll
+                    for (int l = 0; l < 3; ++l) {  // offsets 1, 2, 4 < c (unrolled)
+                        const int off = 1 << l;
+                        if (off < c) {
+                            T o = shfl_up(y, off);
+                            if (qq >= off) y += o;
+                        }
                     }
                     if constexpr (IsInt<T>::value) {
                         E[t] = y - z;
@@ -564,6 +575,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             __syncwarp();
             if (lane == 0) SAM_TRACE(3, tile);
             mbar_arrive(&bar_agg[qs]);
+            if (jsub == cnt - 1) {  // super-tile complete: wake its carry warp (super-tiles round-robin)
+                const int r = i / p.M;
+                // at most one unconsumed phase per barrier: the warp must have taken super-tile r-NCARRY
+                while (cw_taken[r % NCARRY] < r - NCARRY) __nanosleep(32);
+                mbar_arrive(&bar_cw[r % NCARRY]);
+            }
             __syncwarp();
             if (lane == 0) *agg_done = i + 1;
         }
@@ -572,23 +589,20 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         const int npair = s * c;
         for (int r = warp - (NCW + 2);; r += NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;                      // its first iteration
-            // Wait on the aggregator's progress counter first: a carry warp may run several
-            // super-tiles ahead of the aggregator, farther than the mbarrier parity can tell.
+            // Wait for this warp's barrier: the aggregator arrives on it when super-tile r is fully
+            // aggregated, and only after this warp took super-tile r - NCARRY (cw_taken), so the
+            // barrier is never more than one phase ahead and the parity below is unambiguous.
+            const int cw = warp - (NCW + 2);
+            const uint32_t par = (uint32_t)((r / NCARRY) & 1);
             bool ended = false;
-            for (;;) {
-                if (*agg_done > i0) break;
+            while (!mbar_try_wait(&bar_cw[cw], par)) {
                 const int end = *sm_end;
                 if (end >= 0 && i0 >= end) { ended = true; break; }
-                __nanosleep(64);
             }
             if (__any_sync(0xffffffffu, ended)) break;
-            mbar_wait(&bar_agg[i0 % NQ], (uint32_t)((i0 / NQ) & 1));  // acquire the slot data
+            if (lane == 0) cw_taken[cw] = r;
             const int cnt = sub_of[2 * (i0 % NQ) + 1];
             const int il = i0 + cnt - 1;                 // its last iteration
-            if (cnt > 1) {
-                while (*agg_done <= il) __nanosleep(64);
-                mbar_wait(&bar_agg[il % NQ], (uint32_t)((il / NQ) & 1));
-            }
             const int64_t tile = sup_of[i0 % NQ];        // look-back unit: the super-tile
             if (lane == 0) SAM_TRACE(4, tile_of[i0 % NQ]);
             const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate
@@ -988,9 +1002,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                 for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
                 T y = z;
-                for (int off = G; off < 32; off <<= 1) {
-                    T o = shfl_up(y, off);
-                    if (lane >= off) y += o;
+#pragma unroll
+                for (int l = 0; l < 5; ++l) {  // shuffle offsets G, 2G, ... < 32 (unrolled)
+                    const int off = G << l;
+                    if (off < 32) {
+                        T o = shfl_up(y, off);
+                        if (lane >= off) y += o;
+                    }
                 }
                 if constexpr (IsInt<T>::value) {
                     e[t] = y - z;
