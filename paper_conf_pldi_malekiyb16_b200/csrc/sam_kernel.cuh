@@ -127,6 +127,8 @@ struct Params {
     T bq[8][K];           // b_d(q*Uw),     q < c
     T bl[32][K];          // b_d(j*M*U),    j < Wn
     T bsub[8][K];         // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
+    T bks[5][K];          // b_d(2^l*ITEMS) (Kogge-Stone warp scan of thread states, K >= 3)
+    T bkw[3][K];          // b_d(2^l*Uw)    (Kogge-Stone combine of warp states, K >= 3)
 };
 
 // ------------------------------------------------------------------------------------------
@@ -520,27 +522,55 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
                 T E[K], yl[K];
+                if constexpr (K <= 2) {
 #pragma unroll
-                for (int t = 0; t < K; ++t) {
-                    T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
+                    for (int t = 0; t < K; ++t) {
+                        T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
 #pragma unroll
-                    for (int j = 0; j < t; ++j) z += p.bw[t - j] * E[j];
-                    T y = z;
+                        for (int j = 0; j < t; ++j) z += p.bw[t - j] * E[j];
+                        T y = z;
 #pragma unroll
-                    for (int l = 0; l < 3; ++l) {  // offsets 1, 2, 4 < c (unrolled)
+                        for (int l = 0; l < 3; ++l) {  // offsets 1, 2, 4 < c (unrolled)
+                            const int off = 1 << l;
+                            if (off < c) {
+                                T o = shfl_up(y, off);
+                                if (qq >= off) y += o;
+                            }
+                        }
+                        if constexpr (IsInt<T>::value) {
+                            E[t] = y - z;
+                        } else {
+                            T o = shfl_up(y, 1);
+                            E[t] = (qq >= 1) ? o : T(0);
+                        }
+                        yl[t] = y;
+                    }
+                } else {  // Kogge-Stone on k-vectors: yl <- M(2^l Uw) yl_partner + yl
+#pragma unroll
+                    for (int t = 0; t < K; ++t) yl[t] = ok ? wq[(qq * s + mm) * K + t] : T(0);
+#pragma unroll
+                    for (int l = 0; l < 3; ++l) {
                         const int off = 1 << l;
                         if (off < c) {
-                            T o = shfl_up(y, off);
-                            if (qq >= off) y += o;
+                            T o[K];
+#pragma unroll
+                            for (int t = 0; t < K; ++t) o[t] = shfl_up(yl[t], off);
+                            if (qq >= off) {
+#pragma unroll
+                                for (int t = K - 1; t >= 0; --t) {
+                                    T acc2 = yl[t] + o[t];
+#pragma unroll
+                                    for (int j = 0; j < t; ++j) acc2 += p.bkw[l][t - j] * o[j];
+                                    yl[t] = acc2;
+                                }
+                            }
                         }
                     }
-                    if constexpr (IsInt<T>::value) {
-                        E[t] = y - z;
-                    } else {
-                        T o = shfl_up(y, 1);
+#pragma unroll
+                    for (int t = 0; t < K; ++t) {
+                        T o = shfl_up(yl[t], 1);
                         E[t] = (qq >= 1) ? o : T(0);
                     }
-                    yl[t] = y;
                 }
                 __syncwarp();
                 if (ok) {
@@ -993,30 +1023,62 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
                 }
             }
-            // a3: warp scan of thread states (order by order, plain shuffle scans)
-            // e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
-            // z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]
+            // a3: warp scan of thread states.  Orders 1, 2: order by order, plain shuffle scans
+            //   e_{v+1} = M(ITEMS) e_v + a_v  =>  e_{v+1}[t] = e_v[t] + z_v[t],
+            //   z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]      (5k dependent shuffle stages)
+            // Orders >= 3: Kogge-Stone on k-vectors with the carry operator, level l combining
+            //   st <- M(2^l ITEMS) st_partner + st                       (5 dependent stages)
+            if constexpr (K <= 2) {
 #pragma unroll
-            for (int t = 0; t < K; ++t) {
-                T z = acc[t];
+                for (int t = 0; t < K; ++t) {
+                    T z = acc[t];
 #pragma unroll
-                for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
-                T y = z;
+                    for (int j = 0; j < t; ++j) z += p.bc[t - j] * e[j];
+                    T y = z;
 #pragma unroll
-                for (int l = 0; l < 5; ++l) {  // shuffle offsets G, 2G, ... < 32 (unrolled)
+                    for (int l = 0; l < 5; ++l) {  // shuffle offsets G, 2G, ... < 32 (unrolled)
+                        const int off = G << l;
+                        if (off < 32) {
+                            T o = shfl_up(y, off);
+                            if (lane >= off) y += o;
+                        }
+                    }
+                    if constexpr (IsInt<T>::value) {
+                        e[t] = y - z;
+                    } else {
+                        T o = shfl_up(y, G);
+                        e[t] = (lane >= G) ? o : T(0);
+                    }
+                    if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
+                }
+            } else {
+                T st[K];
+#pragma unroll
+                for (int t = 0; t < K; ++t) st[t] = acc[t];
+#pragma unroll
+                for (int l = 0; l < 5; ++l) {
                     const int off = G << l;
                     if (off < 32) {
-                        T o = shfl_up(y, off);
-                        if (lane >= off) y += o;
+                        T o[K];
+#pragma unroll
+                        for (int t = 0; t < K; ++t) o[t] = shfl_up(st[t], off);
+                        if (lane >= off) {
+#pragma unroll
+                            for (int t = K - 1; t >= 0; --t) {
+                                T acc2 = st[t] + o[t];
+#pragma unroll
+                                for (int j = 0; j < t; ++j) acc2 += p.bks[l][t - j] * o[j];
+                                st[t] = acc2;
+                            }
+                        }
                     }
                 }
-                if constexpr (IsInt<T>::value) {
-                    e[t] = y - z;
-                } else {
-                    T o = shfl_up(y, G);
+#pragma unroll
+                for (int t = 0; t < K; ++t) {
+                    T o = shfl_up(st[t], G);
                     e[t] = (lane >= G) ? o : T(0);
+                    if (v == Pw - 1) wq[(q * s + m) * K + t] = st[t];  // warp aggregate of lane m
                 }
-                if (v == Pw - 1) wq[(q * s + m) * K + t] = y;  // warp aggregate of lane m
             }
             mbar_arrive(&bar_p1[qs]);  // warp states ready; P1 buffer free for the producer
         };

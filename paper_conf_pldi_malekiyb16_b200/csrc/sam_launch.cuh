@@ -148,6 +148,8 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
     for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, p.bl[j]);
     for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, p.bsub[j]);
+    for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * Cfg<T>::ITEMS, K, p.bks[l]);
+    for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, p.bkw[l]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
