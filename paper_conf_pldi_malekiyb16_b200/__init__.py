@@ -24,7 +24,8 @@ SAM_I32, SAM_I64, SAM_F32, SAM_F64 = 0, 1, 2, 3
 _STATUS = {0: "SAM_OK", -1: "SAM_ERR_INVALID_ARG", -2: "SAM_ERR_UNSUPPORTED", -3: "SAM_ERR_CUDA",
            -4: "SAM_ERR_OOM", -5: "SAM_ERR_INTERNAL"}
 
-LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libsam.so")
+LIB_PATH = os.environ.get("SAM_LIB_PATH") or \
+    os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libsam.so")  # override: experiments
 _lib = None
 
 

@@ -60,17 +60,24 @@ template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
 //   <= 8 B : 3 local-scan buffers, 3 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
 //   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
 //   larger : 3 + 2 buffers, pending states in registers (LAG = 4), super-tiles of 2
+// (SAM_LAG_SMALL / SAM_SPLIT_MIN_K: compile-time overrides for experiments, tools/build_variant.py)
+#ifndef SAM_LAG_SMALL
+#define SAM_LAG_SMALL 12
+#endif
+#ifndef SAM_SPLIT_MIN_K
+#define SAM_SPLIT_MIN_K 2
+#endif
 template <typename T, int K> struct Lag {
     static constexpr int SB = K * (int)sizeof(T);
     static constexpr bool SMEM = SB <= 16;           // pending local states in shared memory
-    static constexpr int LAG = SB <= 8 ? 12 : (SB <= 16 ? 8 : 4);
+    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? 12 : (SB <= 16 ? 8 : 4));
     static constexpr int MMAX = SB <= 8 ? 4 : 2;     // max tiles per super-tile (look-back unit)
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
     static constexpr int NB2 = SB <= 8 ? 4 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = SMEM && K >= 2;
+    static constexpr bool SPLIT = SMEM && K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
@@ -109,6 +116,7 @@ struct Params {
     int U, T_, Uw;
     int inclusive;
     int store_mode;
+    int claim_slack;      // experiments: extra claimed-but-blocked tiles (0 = never block a local scan)
     const T* seed;        // [s][K] state before the stream per global lane, or null
     T* final_state;       // [s][K] or null
     int64_t last_e[MAXS]; // virtual index of lane m's last element, -1 if none
@@ -436,7 +444,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 bulk_commit();  // one group per stored iteration (possibly empty)
             };
             int j1 = 0, j2 = 0, j3 = 0, jend = -1;
-            unsigned long long next_claim = atomicAdd(p.tile_ctr, 1ull);
+            unsigned long long claimed = 0;
+            bool claim_pending = false;
             int64_t cur_sup = -1;
             int cur_j = 0, cur_cnt = 0;
             for (;;) {
@@ -461,14 +470,24 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     ++j2;
                     continue;
                 }
-                // (3) claim and load a new tile (buffer free, at most PF unscanned, slot free).  The
-                // claim's atomic was issued one step earlier, so its round trip is off this path.
-                if (jend < 0 && j3 > j1 - NQ &&
+                // (3) claim and load a new tile (buffer free, at most PF unscanned, pending-state slot
+                // free: tile j1's local scan needs the carry application of j1 - LAG done, and a
+                // loaded tile must never wait for that -- its aggregate gates every later tile's
+                // look-back).  A super-tile is claimed only once it can be loaded at once: a claimed
+                // but unloaded super-tile stalls every later look-back on the GPU.  The atomic is
+                // issued when the load conditions hold and consumed on the next pass through this
+                // branch, so stores and reloads that become ready meanwhile are not held up by it.
+                if (jend < 0 && j1 < j3 + LAG + p.claim_slack &&
                     (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
                     (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
                     if (cur_j == cur_cnt) {  // start the next super-tile
-                        cur_sup = (int64_t)next_claim;
-                        next_claim = atomicAdd(p.tile_ctr, 1ull);
+                        if (!claim_pending) {
+                            claimed = atomicAdd(p.tile_ctr, 1ull);
+                            claim_pending = true;
+                            continue;
+                        }
+                        claim_pending = false;
+                        cur_sup = (int64_t)claimed;
                         cur_j = 0;
                         cur_cnt = 0;
                         if ((uint64_t)cur_sup < p.num_super) {
@@ -935,18 +954,29 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 auto items = [&](auto excl_tag, auto slow_tag) {
                     constexpr bool EXCL = decltype(excl_tag)::value;
                     constexpr bool SLOW = decltype(slow_tag)::value;
+                    // all ITEMS loads first: interleaving them with the (possibly aliasing, as far
+                    // as the compiler knows) stores would serialise every item on an smem round trip
+                    T xv[ITEMS];
 #pragma unroll
                     for (int i = 0; i < ITEMS; ++i) {
                         const int el = base_loc + i * s;
-                        T x;
+                        if constexpr (SLOW) {
+                            const uint64_t ve = e0 + el;
+                            const bool valid = !masked || (ve >= p.h && ve < p.h + p.n);
+                            xv[i] = valid ? xs[el] : T(0);
+                        } else {
+                            xv[i] = xs[el];
+                        }
+                    }
+#pragma unroll
+                    for (int i = 0; i < ITEMS; ++i) {
+                        const int el = base_loc + i * s;
+                        const T x = xv[i];
                         bool valid = true;
                         uint64_t ve = 0;
                         if constexpr (SLOW) {
                             ve = e0 + el;
                             valid = !masked || (ve >= p.h && ve < p.h + p.n);
-                            x = valid ? xs[el] : T(0);
-                        } else {
-                            x = xs[el];
                         }
                         y[0] += x;
 #pragma unroll

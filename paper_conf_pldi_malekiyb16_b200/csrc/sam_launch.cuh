@@ -105,6 +105,10 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     p.Pw = geo.Pw; p.W = geo.W; p.Wn = geo.Wn; p.U = geo.U; p.T_ = geo.T; p.Uw = geo.Uw;
     p.inclusive = a.inclusive;
     p.store_mode = a.store_mode;
+    if (const char* env = getenv("SAM_CLAIM_SLACK")) {  // experiments (ring slots allow at most 2)
+        const int v = atoi(env);
+        p.claim_slack = v < 0 ? 0 : (v > 2 ? 2 : v);
+    }
     p.seed = (const T*)a.seed;
     p.final_state = (T*)a.final_state;
     for (int m = 0; m < MAXS; ++m) {

@@ -26,3 +26,10 @@ d = (t[:-1, 3] - t[1:, 3]) / 1e3
 print(f"agg(t-1) - agg(t)        {q(d)}")
 d = (t[:-1, 5] - t[1:, 3]) / 1e3
 print(f"incl(t-1) - agg(t)       {q(d)}")
+# parked footprint: tiles between claim (HBM load issued) and carry application start (L2 reload done)
+tile_bytes = x.element_size() * (n // max(1, len(t)))
+ev = np.concatenate([np.stack([t[:, 0], np.ones(len(t))], 1), np.stack([t[:, 6], -np.ones(len(t))], 1)])
+ev = ev[np.argsort(ev[:, 0], kind="stable")]
+occ = np.cumsum(ev[:, 1])
+print(f"parked tiles: p50 {np.percentile(occ, 50):.0f}  p90 {np.percentile(occ, 90):.0f}  max {occ.max():.0f}"
+      f"  (~{np.percentile(occ, 50) * tile_bytes / 2**20:.1f} / {occ.max() * tile_bytes / 2**20:.1f} MiB)")
