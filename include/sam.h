@@ -134,10 +134,11 @@ const char* sam_version(void);
 int sam_release_workspaces(void);
 /* Kernel launches issued by this library on the calling process since load (for bench). */
 uint64_t sam_launch_count(void);
-/* Diagnostics: when trace_dev (device memory, >= 8 * tiles u64) is non-NULL, subsequent scan
- * launches record %globaltimer at 8 pipeline events of every tile: [tile][claim, P1 start,
- * P1 done, aggregate published, look-back start, inclusive published, carry applied, stored].
- * NULL turns tracing off. */
+/* Diagnostics: when trace_dev (device memory, >= 16 * tiles u64, zeroed) is non-NULL, subsequent
+ * scan launches record %globaltimer at pipeline events of every tile: [tile][claim, P1 start,
+ * P1 done, aggregate published, look-back start, inclusive published, carry applied, stored,
+ * first poll issued, first poll returned, look-back done, #polls, stop = own previous unit, ...]
+ * (look-back fields on the first tile of each look-back unit).  NULL turns tracing off. */
 int sam_debug_set_trace(void* trace_dev);
 
 #ifdef __cplusplus

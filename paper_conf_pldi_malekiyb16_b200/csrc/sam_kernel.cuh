@@ -64,6 +64,15 @@ template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
 #ifndef SAM_LAG_SMALL
 #define SAM_LAG_SMALL 12
 #endif
+// SAM_EARLY_RELOAD: re-fetch a tile into a carry buffer as soon as its local scan is done (the
+// carry application then also waits for the carry) instead of once its carry is known
+#ifndef SAM_EARLY_RELOAD
+#define SAM_EARLY_RELOAD 0
+#endif
+// SAM_LB_EARLY: start a super-tile's carry fold before its own aggregate is complete
+#ifndef SAM_LB_EARLY
+#define SAM_LB_EARLY 0
+#endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
 #endif
@@ -97,8 +106,8 @@ enum StoreMode { STORE_BULK = 0, STORE_STRIPED = 1, STORE_NONE = 2 };
 template <typename T> struct TagW { static constexpr int W = sizeof(T) == 4 ? 1 : 2; };
 // look-back window rows per round trip (carry-warp register budget: V*K*2W <= 16 words per lane)
 template <typename T, int K> struct LB {
-    static constexpr int W2 = 2 * TagW<T>::W;
-    static constexpr int V0 = 16 / (K * W2);
+    static constexpr int W1 = TagW<T>::W;
+    static constexpr int V0 = 16 / (K * W1);
     static constexpr int V = V0 < 1 ? 1 : (V0 > 16 ? 16 : V0);
 };
 
@@ -217,7 +226,7 @@ __device__ __forceinline__ unsigned long long globaltimer() {
 // diagnostics: record event ev (0..7) of tile `tile` when tracing is on
 #define SAM_TRACE(ev, tile)                                                        \
     do {                                                                           \
-        if (p.trace) p.trace[(size_t)(tile) * 8 + (ev)] = globaltimer();           \
+        if (p.trace) p.trace[(size_t)(tile) * 16 + (ev)] = globaltimer();          \
     } while (0)
 __device__ __forceinline__ uint64_t policy_evict_last() {
     uint64_t p;
@@ -228,6 +237,11 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     uint64_t p;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+    unsigned long long a;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(a) : "l"(p) : "memory");
+    return a;
 }
 __device__ __forceinline__ void ld_relaxed_v2(const unsigned long long* p, unsigned long long& a,
                                               unsigned long long& b) {
@@ -258,15 +272,15 @@ template <> struct Bits<double> {
 
 // publish value v of slot (tile, m, t), half = 0 (aggregate) or 1 (inclusive)
 template <typename T>
-__device__ __forceinline__ void put_tagged(unsigned long long* slot, int half, uint32_t tag, T v) {
+__device__ __forceinline__ void put_tagged(unsigned long long* slot, uint32_t tag, T v) {
     constexpr int W = TagW<T>::W;
     const uint64_t b = Bits<T>::to(v);
     const uint64_t hi = (uint64_t)tag << 32;
     if constexpr (W == 1) {
-        st_relaxed_u64(slot + half, hi | (b & 0xffffffffull));
+        st_relaxed_u64(slot, hi | (b & 0xffffffffull));
     } else {
-        st_relaxed_u64(slot + 2 * half, hi | (b & 0xffffffffull));
-        st_relaxed_u64(slot + 2 * half + 1, hi | (b >> 32));
+        st_relaxed_u64(slot, hi | (b & 0xffffffffull));
+        st_relaxed_u64(slot + 1, hi | (b >> 32));
     }
 }
 
@@ -304,15 +318,17 @@ struct Smem {
     static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
     static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
     static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
-    static constexpr int OFF_TAG = OFF_SUB + NQ * 8;                     // u32 tag, i32 end, i32 agg progress
-    static constexpr int OFF_CW = OFF_TAG + 16;                          // NCARRY x i32 super-tile taken
+    static constexpr int OFF_TAG = OFF_SUB + NQ * 8;                     // u32 tag, i32 end, i32 agg progress, i32 p2, i32 claims
+    static constexpr int OFF_CW = OFF_TAG + 32;                          // NCARRY x i32 super-tile taken
     static constexpr int OFF_WQ = (OFF_CW + 4 * NCARRY + 15) / 16 * 16;  // NQ x [64][K]
     static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
     static constexpr int OFF_LP = OFF_LA + NQ * LA * (int)sizeof(T);     // NQ x [8][K] in-super prefix
     static constexpr int OFF_BT = OFF_LP + NQ * LA * (int)sizeof(T);     // [K][32]
     static constexpr int OFF_BL = OFF_BT + K * 32 * (int)sizeof(T);      // [NBL][K]
     static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
-    static constexpr int OFF_EQ = OFF_BQ + 8 * K * (int)sizeof(T);       // [ELAG][TILE_THREADS][K]
+    static constexpr int HOB = 16 + MAXS * K * (int)sizeof(T);           // hand-off entry: i32 r, pad, [MAXS][K]
+    static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
+    static constexpr int OFF_EQ = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;  // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
 };
 
@@ -330,7 +346,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int LAG = S::LAG;
     constexpr bool ESMEM = Lag<T, K>::SMEM;
     constexpr int PF = Lag<T, K>::PF;
-    constexpr int W2 = 2 * TagW<T>::W;  // tagged words per slot (aggregate + inclusive)
+    constexpr int W1 = TagW<T>::W;      // tagged words per published value
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
@@ -383,6 +399,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         for (int w = 0; w < NCARRY; ++w) {
             mbar_init(&bar_cw[w], 32);
             cw_taken[w] = -1;
+            *(volatile int*)(smem + S::OFF_HO + w * S::HOB) = -1;
         }
         fence_mbar_init();
         *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
@@ -444,10 +461,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 bulk_commit();  // one group per stored iteration (possibly empty)
             };
             int j1 = 0, j2 = 0, j3 = 0, jend = -1;
-            unsigned long long claimed = 0;
-            bool claim_pending = false;
             int64_t cur_sup = -1;
-            int cur_j = 0, cur_cnt = 0;
+            int cur_j = 0, cur_cnt = 0, nsup = 0;
             for (;;) {
                 // (1) store the oldest iteration whose carry application is done
                 if (j3 < j2 && mbar_test(&bar_stored2[j3 % NB2], (uint32_t)((j3 / NB2) & 1))) {
@@ -458,7 +473,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
                 // (2) reload (from L2) the next tile whose carry is known, into a free carry buffer
                 if (j2 < j1 && j2 - j3 < NB2 &&
-                    mbar_test(&bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
+                    mbar_test(SAM_EARLY_RELOAD ? &bar_p1[j2 % NQ] : &bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
                     // groups committed after the store that last used this buffer (iteration j2-NB2)
                     const int later = j3 - 1 - (j2 - NB2);
                     if (later <= 0) bulk_wait_read<0>();
@@ -470,24 +485,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     ++j2;
                     continue;
                 }
-                // (3) claim and load a new tile (buffer free, at most PF unscanned, pending-state slot
-                // free: tile j1's local scan needs the carry application of j1 - LAG done, and a
-                // loaded tile must never wait for that -- its aggregate gates every later tile's
-                // look-back).  A super-tile is claimed only once it can be loaded at once: a claimed
-                // but unloaded super-tile stalls every later look-back on the GPU.  The atomic is
-                // issued when the load conditions hold and consumed on the next pass through this
-                // branch, so stores and reloads that become ready meanwhile are not held up by it.
+                // (3) load the next tile of this CTA's static schedule (super-tiles b, b+P, ...) once
+                // a buffer is free, at most PF tiles are unscanned and a pending-state slot is free
+                // (tile j1's local scan needs the carry application of j1 - LAG done, and a loaded
+                // tile must never wait for that -- its aggregate gates the other CTAs' carries)
                 if (jend < 0 && j1 < j3 + LAG + p.claim_slack &&
                     (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
                     (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
                     if (cur_j == cur_cnt) {  // start the next super-tile
-                        if (!claim_pending) {
-                            claimed = atomicAdd(p.tile_ctr, 1ull);
-                            claim_pending = true;
-                            continue;
-                        }
-                        claim_pending = false;
-                        cur_sup = (int64_t)claimed;
+                        cur_sup = (int64_t)blockIdx.x + (int64_t)nsup * gridDim.x;
+                        ++nsup;
                         cur_j = 0;
                         cur_cnt = 0;
                         if ((uint64_t)cur_sup < p.num_super) {
@@ -613,8 +620,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                             for (int t = 0; t < K; ++t) {
                                 la[mm * K + t] = Pref[ch][t];  // super-tile aggregate
-                                if (sup > 0) {  // a4: publish it
-                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W2, 0, tag, Pref[ch][t]);
+                                {  // a4: publish it
+                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W1, tag, Pref[ch][t]);
                                 }
                             }
                         }
@@ -634,31 +641,34 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if (lane == 0) *agg_done = i + 1;
         }
     } else if (warp >= NCW + 2) {
-        // =========================== carry warps: decoupled look-back, inclusive states ==========
+        // =========================== carry warps: carry-in of each super-tile ===================
+        // a5, SAM's carry scheme on a static schedule: CTA b owns super-tiles
+        // b, b+P, b+2P, ... (P = gridDim.x, all CTAs co-resident: cooperative launch).  The carry
+        // into super-tile S is this CTA's own inclusive state after S-P (kept in shared memory)
+        // advanced over the P-1 aggregates published by the other CTAs in between:
+        //   C_S = M((P-1) US) I_{S-P} + sum_{j=S-P+1}^{S-1} M((S-1-j) US) A_j
+        // read in windows of Wn*V super-tiles, one L2 round trip each (no inclusive chain
+        // between CTAs, hence no serial latency).
         const int npair = s * c;
-        for (int r = warp - (NCW + 2);; r += NCARRY) {  // this CTA's r-th super-tile
-            const int i0 = r * p.M;                      // its first iteration
+        const int cw = warp - (NCW + 2);
+        for (int r = cw;; r += NCARRY) {  // this CTA's r-th super-tile
+            const int i0 = r * p.M;       // its first iteration
+            const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
+            if ((uint64_t)tile >= p.num_super) break;
+            const int64_t Sprev = r == 0 ? (int64_t)-1 : tile - gridDim.x;
+            const bool lane_ok = lane < s;
+            const int ml = lane_ok ? lane : 0;
+#if !SAM_LB_EARLY
             // Wait for this warp's barrier: the aggregator arrives on it when super-tile r is fully
             // aggregated, and only after this warp took super-tile r - NCARRY (cw_taken), so the
             // barrier is never more than one phase ahead and the parity below is unambiguous.
-            const int cw = warp - (NCW + 2);
-            const uint32_t par = (uint32_t)((r / NCARRY) & 1);
-            bool ended = false;
-            while (!mbar_try_wait(&bar_cw[cw], par)) {
-                const int end = *sm_end;
-                if (end >= 0 && i0 >= end) { ended = true; break; }
-            }
-            if (__any_sync(0xffffffffu, ended)) break;
+            mbar_wait(&bar_cw[cw], (uint32_t)((r / NCARRY) & 1));
+            __syncwarp();
             if (lane == 0) cw_taken[cw] = r;
-            const int cnt = sub_of[2 * (i0 % NQ) + 1];
-            const int il = i0 + cnt - 1;                 // its last iteration
-            const int64_t tile = sup_of[i0 % NQ];        // look-back unit: the super-tile
-            if (lane == 0) SAM_TRACE(4, tile_of[i0 % NQ]);
-            const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate
-            const bool lane_ok = lane < s;
-            const int ml = lane_ok ? lane : 0;
+#endif
+            if (lane == 0) SAM_TRACE(4, tile * p.M);
 
-            // seed of virtual tile -1 for lane mm: M(-1) applied for lanes before the phase
+            // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, T* out) {
                 if (p.seed) {
 #pragma unroll
@@ -673,104 +683,92 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
             };
 
-            constexpr int INF = 1 << 30;
             T C[K];
-            if (tile == 0) {
-                seed_of(ml, C);
-            } else {
-                // a5: lane = (jl, mlb); window row vv holds predecessor distance d = jl + Wn*vv
+            {
+                // lane = (jl, mlb); window row vv holds the super-tile at distance d = jl + Wn*vv
+                // before basei; rows beyond Sprev hold nothing, the row AT Sprev holds this CTA's
+                // previous inclusive state (or, for r = 0, the seed of virtual super-tile -1)
                 const int Wn = p.Wn;
                 const int jl = lane / s, mlb = lane - jl * s;
                 const bool active = jl < Wn;
-                const unsigned smask = (1u << s) - 1u;
                 T total[K], Pm[K];
 #pragma unroll
                 for (int t = 0; t < K; ++t) { total[t] = T(0); Pm[t] = (t == 0) ? T(1) : T(0); }
                 int64_t basei = tile - 1;
                 bool first = true;
+                int npoll = 0;
                 for (;;) {
-                    unsigned long long w[V][K][W2];
-                    int st[V];  // 0 invalid, 1 aggregate valid, 2 inclusive valid, 3 ignored
+                    unsigned long long w[V][K][W1];
+                    int st[V];  // 0 pending, 1 aggregate valid, 2 previous inclusive / seed, 3 nothing
 #pragma unroll
                     for (int vv = 0; vv < V; ++vv) {
                         const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                        st[vv] = !active ? 3 : (idx == -1 ? 2 : (idx < -1 ? 3 : 0));
+                        st[vv] = !active ? 3 : (idx > Sprev ? 0 : (idx == Sprev ? 2 : 3));
                     }
-                    int dI;
                     for (;;) {
+                        if (p.trace && lane == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
+                        bool pend = false;
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
                                 const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                                const unsigned long long* src = p.carry + ((size_t)idx * s + mlb) * K * W2;
-                                bool ag = true, in = true;
+                                const unsigned long long* src = p.carry + ((size_t)idx * s + mlb) * K * W1;
+                                bool ok = true;
 #pragma unroll
                                 for (int t = 0; t < K; ++t) {
-                                    if constexpr (W2 == 2) {
-                                        ld_relaxed_v2(src + t * 2, w[vv][t][0], w[vv][t][1]);
-                                        ag &= (uint32_t)(w[vv][t][0] >> 32) == tag;
-                                        in &= (uint32_t)(w[vv][t][1] >> 32) == tag;
+                                    if constexpr (W1 == 1) {
+                                        w[vv][t][0] = ld_relaxed_u64(src + t);
+                                        ok &= (uint32_t)(w[vv][t][0] >> 32) == tag;
                                     } else {
-                                        ld_relaxed_v2(src + t * 4, w[vv][t][0], w[vv][t][1]);
-                                        ld_relaxed_v2(src + t * 4 + 2, w[vv][t][2], w[vv][t][3]);
-                                        ag &= (uint32_t)(w[vv][t][0] >> 32) == tag &&
+                                        ld_relaxed_v2(src + 2 * t, w[vv][t][0], w[vv][t][1]);
+                                        ok &= (uint32_t)(w[vv][t][0] >> 32) == tag &&
                                               (uint32_t)(w[vv][t][1] >> 32) == tag;
-                                        in &= (uint32_t)(w[vv][t][2] >> 32) == tag &&
-                                              (uint32_t)(w[vv][t][3] >> 32) == tag;
                                     }
                                 }
-                                st[vv] = in ? 2 : (ag ? 1 : 0);
+                                st[vv] = ok ? 1 : 0;
+                                pend |= !ok;
                             }
                         }
-                        // nearest tile whose s lanes are all inclusive-valid, nearest invalid one
-                        dI = INF;
-                        int dX = INF;
-#pragma unroll
-                        for (int vv = 0; vv < V; ++vv) {
-                            const unsigned bv = __ballot_sync(0xffffffffu, st[vv] >= 1);
-                            const unsigned bi = __ballot_sync(0xffffffffu, st[vv] == 2);
-                            unsigned gv = bv, gi = bi;
-                            if (s > 1) {
-                                gv = gi = 0;
-                                for (int j = 0; j < Wn; ++j) {
-                                    if (((bv >> (j * s)) & smask) == smask) gv |= 1u << j;
-                                    if (((bi >> (j * s)) & smask) == smask) gi |= 1u << j;
-                                }
-                            }
-                            const unsigned full = (Wn == 32) ? 0xffffffffu : ((1u << Wn) - 1u);
-                            const unsigned inv = ~gv & full;
-                            if (gi && dI == INF) dI = Wn * vv + (__ffs(gi) - 1);
-                            if (inv && dX == INF) dX = Wn * vv + (__ffs(inv) - 1);
-                        }
-                        if (dI < dX || (dX == INF && dI == INF)) break;
+                        if (p.trace && lane == 0 && npoll == 0) SAM_TRACE(9, tile * p.M);
+                        ++npoll;
+                        if (!__any_sync(0xffffffffu, pend)) break;
                     }
-                    // fold: d < dI aggregates, d == dI inclusive.  This lane's tiles sit at
-                    // d = jl + Wn*vv, so by Horner in vv:
-                    //   sum_vv M((jl + Wn vv) U) X_vv = M(jl U) (X_0 + M(Wn U)(X_1 + M(Wn U)(X_2 + ...)))
+                    const bool last = basei - (int64_t)Wn * V < Sprev;  // this window holds Sprev
+                    if (p.trace && lane == 0 && last) {
+                        SAM_TRACE(10, tile * p.M);
+                        p.trace[(size_t)(tile * p.M) * 16 + 11] = npoll;
+                    }
+                    if (last && Sprev >= 0) {  // previous inclusive state: wait for its hand-off entry
+                        const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
+                        while (*rt != r - 1) __nanosleep(20);
+                        __syncwarp();
+                    }
+                    // fold.  This lane's rows sit at d = jl + Wn*vv, so by Horner in vv:
+                    //   sum_vv M((jl + Wn vv) US) X_vv = M(jl US) (X_0 + M(Wn US)(X_1 + M(Wn US)(X_2 + ...)))
                     T Y[K];
 #pragma unroll
                     for (int t = 0; t < K; ++t) Y[t] = T(0);
 #pragma unroll
                     for (int vv = V - 1; vv >= 0; --vv) {
-                        const int d = jl + Wn * vv;
                         T X[K];
 #pragma unroll
                         for (int t = 0; t < K; ++t) X[t] = T(0);
-                        if (active && d <= dI && st[vv] != 3) {
-                            const int64_t idx = basei - d;
-                            if (idx == -1) {
+                        if (st[vv] == 1) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) {
+                                if constexpr (W1 == 1) {
+                                    X[t] = Bits<T>::from(w[vv][t][0] & 0xffffffffull);
+                                } else {
+                                    X[t] = Bits<T>::from((w[vv][t][0] & 0xffffffffull) | (w[vv][t][1] << 32));
+                                }
+                            }
+                        } else if (st[vv] == 2) {
+                            if (Sprev < 0) {
                                 seed_of(mlb, X);
                             } else {
-                                const int half = (d == dI) ? 1 : 0;
+                                const T* hv = (const T*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
 #pragma unroll
-                                for (int t = 0; t < K; ++t) {
-                                    if constexpr (W2 == 2) {
-                                        X[t] = Bits<T>::from(w[vv][t][half] & 0xffffffffull);
-                                    } else {
-                                        X[t] = Bits<T>::from((w[vv][t][2 * half] & 0xffffffffull) |
-                                                             (w[vv][t][2 * half + 1] << 32));
-                                    }
-                                }
+                                for (int t = 0; t < K; ++t) X[t] = hv[mlb * K + t];
                             }
                         }
                         if (vv == V - 1) {
@@ -778,7 +776,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             for (int t = 0; t < K; ++t) Y[t] = X[t];
                         } else {
 #pragma unroll
-                            for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn U) Y + X
+                            for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn US) Y + X
                                 T acc2 = Y[t] + X[t];
 #pragma unroll
                                 for (int j = 0; j < t; ++j) acc2 += p.bwn[t - j] * Y[j];
@@ -786,7 +784,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             }
                         }
                     }
-                    if (active) {  // Y <- M(jl U) Y
+                    if (active) {  // Y <- M(jl US) Y
 #pragma unroll
                         for (int t = K - 1; t >= 1; --t) {
                             T acc2 = Y[t];
@@ -802,7 +800,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             if (jl + off < Wn) Y[t] += o;
                         }
                     }
-                    // lanes jl == 0 hold this round trip's sum; total += M(offset) Y
+                    // lanes jl == 0 hold this window's sum; total += M(offset) Y
                     if (first) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) total[t] = Y[t];
@@ -815,8 +813,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             total[t] += acc2;
                         }
                     }
-                    if (dI < INF) break;
-                    {   // Pm <- Pm * M(Wn*V*U)  (truncated polynomial product)
+                    if (last) break;
+                    {   // Pm <- Pm * M(Wn*V*US)  (truncated polynomial product)
                         T np[K];
 #pragma unroll
                         for (int d = 0; d < K; ++d) {
@@ -835,15 +833,36 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 for (int t = 0; t < K; ++t) C[t] = total[t];
             }
 
-            // publish the inclusive state of this super-tile: M(M U) C + A
-            if ((uint64_t)tile + 1 < p.num_super && lane_ok) {
-                unsigned long long* const carry_tile = p.carry + (size_t)tile * s * K * W2;
+#if SAM_LB_EARLY
+            mbar_wait(&bar_cw[cw], (uint32_t)((r / NCARRY) & 1));
+            __syncwarp();
+            if (lane == 0) cw_taken[cw] = r;
+#endif
+            const int cnt = sub_of[2 * (i0 % NQ) + 1];
+            const int il = i0 + cnt - 1;                 // its last iteration
+            const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate
+            // hand the inclusive state M(M US) C + A to this CTA's next super-tile (in order
+            // r-1 -> r: slot r % NCARRY is free once r-1's entry exists, r-1 having waited for r-2 ...)
+            if ((uint64_t)tile + gridDim.x < p.num_super) {
+                if (r > 0) {
+                    const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
+                    while (*rt != r - 1) __nanosleep(20);
+                }
+                __syncwarp();
+                unsigned char* ho = smem + S::OFF_HO + (r % NCARRY) * S::HOB;
+                if (lane_ok) {
 #pragma unroll
-                for (int t = 0; t < K; ++t) {
-                    T acc2 = C[t] + la[ml * K + t];
+                    for (int t = 0; t < K; ++t) {
+                        T acc2 = C[t] + la[ml * K + t];
 #pragma unroll
-                    for (int j = 0; j < t; ++j) acc2 += p.bus[t - j] * C[j];
-                    put_tagged<T>(carry_tile + (lane * K + t) * W2, 1, tag, acc2);
+                        for (int j = 0; j < t; ++j) acc2 += p.bus[t - j] * C[j];
+                        ((T*)(ho + 16))[lane * K + t] = acc2;
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    __threadfence_block();
+                    *(volatile int*)ho = r;
                 }
             }
             // each sub-tile j: C_j = M(j U) C + P_j, then per-warp incoming states
@@ -1132,6 +1151,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 for (int i = 0;; ++i) {
                     const int b2 = i % NB2;
                     if (!wait_or_end(&bar_full2[b2], (uint32_t)((i / NB2) & 1), i)) break;
+                    if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                     T e[K];
 #pragma unroll
                     for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
@@ -1178,9 +1198,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     const int i = p2_next;
                     const int b2 = i % NB2;
                     const uint32_t par = (uint32_t)((i / NB2) & 1);
-                    const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)mbar_test(&bar_full2[b2], par) : 0, 0);
+                    const bool ready = __shfl_sync(0xffffffffu, lane == 0 ? (int)(mbar_test(&bar_full2[b2], par) &&
+                        (!SAM_EARLY_RELOAD || mbar_test(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1)))) : 0, 0);
                     if (ready) {
                         mbar_wait(&bar_full2[b2], par);
+                        if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                         T e[K];
                         if constexpr (ESMEM) {
 #pragma unroll

@@ -131,8 +131,12 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
         if (m > (uint64_t)Lag<T, K>::MMAX) m = Lag<T, K>::MMAX;
         if (const char* env = getenv("SAM_SUPER_TILE")) {  // experiments: force a smaller super-tile
             const int f = atoi(env);
-            if (f >= 1 && (uint64_t)f < m) m = (uint64_t)f;
+            if (f >= 1 && f <= 8) m = (uint64_t)f;
         }
+        // a super-tile is aggregated before its carry is known: at most LAG/2 tiles per unit
+        // keep two units in flight per CTA (LAG bounds the tiles between load and carry application)
+        const uint64_t mlag = Lag<T, K>::LAG / 2 > 1 ? Lag<T, K>::LAG / 2 : 1;
+        if (m > mlag) m = mlag;
         p.M = (int)m;
         p.num_super = (p.num_tiles + m - 1) / m;
     }
@@ -156,12 +160,25 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, p.bkw[l]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
+    // Static schedule (CTA b owns super-tiles b, b+P, ...): every CTA waits on aggregates of the
+    // others, so all P CTAs must be co-resident -- a cooperative launch guarantees it (or fails).
     uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
-    if (grid > p.num_tiles) grid = p.num_tiles;
+    if (grid > p.num_super) grid = p.num_super;
     if (grid < 1) grid = 1;
-    sam_scan_kernel<T, K><<<(unsigned)grid, (Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32, S::BYTES, a.stream>>>(p);
-    if (launches) ++*launches;
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg;
+    memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3((Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32);
+    cfg.dynamicSmemBytes = S::BYTES;
+    cfg.stream = a.stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sam_scan_kernel<T, K>, p);
+    if (launches && e == cudaSuccess) ++*launches;
+    return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 template <typename T>

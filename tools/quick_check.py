@@ -6,7 +6,7 @@ import oracle, synth
 import paper_conf_pldi_malekiyb16_b200 as S
 
 def check(dt, n, k, s, incl):
-    xn = synth.make(n, dt, "uniform", seed=n + k * 8 + s)
+    xn = synth.make(n, dt, "uniform" if dt in ("i32", "i64") else "unif01", seed=n + k * 8 + s)
     x = torch.from_numpy(xn).cuda()
     y = S.scan(x, k, s, incl); torch.cuda.synchronize()
     ref = oracle.scan(xn, k, s, incl)[0]

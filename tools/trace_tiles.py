@@ -8,13 +8,14 @@ n = 1 << logn
 x = synth.make_torch(n, dt, "uniform", device="cuda"); y = torch.empty_like(x)
 for _ in range(3): S.scan(x, k, s, True, out=y)
 torch.cuda.synchronize()
-tr = torch.zeros(8 * (n // 1000 + 16), dtype=torch.int64, device="cuda")
+tr = torch.zeros(16 * (n // 1000 + 16), dtype=torch.int64, device="cuda")
 S.lib().sam_debug_set_trace(ctypes.c_void_p(tr.data_ptr()))
 S.scan(x, k, s, True, out=y); torch.cuda.synchronize()
 S.lib().sam_debug_set_trace(None)
-t = tr.cpu().numpy().reshape(-1, 8)
+t = tr.cpu().numpy().reshape(-1, 16)
 t = t[t[:, 0] > 0]
-t = t - t[:, 0].min()
+extra = t[:, 8:].copy()
+t = t[:, :8] - t[:, 0].min()
 names = ["claim", "p1start", "p1done", "aggpub", "lbstart", "inclpub", "p2start", "stored"]
 print(f"{dt} 2^{logn} k={k} s={s}: tiles {len(t)}  span {t.max()/1e3:.1f} us  rate {len(t)/(t.max()/1e3):.1f} tiles/us")
 def q(a): return " ".join(f"{np.percentile(a, pp):7.2f}" for pp in (10, 50, 90, 99))
@@ -33,3 +34,6 @@ ev = ev[np.argsort(ev[:, 0], kind="stable")]
 occ = np.cumsum(ev[:, 1])
 print(f"parked tiles: p50 {np.percentile(occ, 50):.0f}  p90 {np.percentile(occ, 90):.0f}  max {occ.max():.0f}"
       f"  (~{np.percentile(occ, 50) * tile_bytes / 2**20:.1f} / {occ.max() * tile_bytes / 2**20:.1f} MiB)")
+lb = extra[extra[:, 0] > 0]
+if len(lb):
+    print(f"look-back units {len(lb)}: first poll RTT {q((lb[:,1]-lb[:,0])/1e3)}  loop {q((lb[:,2]-lb[:,0])/1e3)}  polls {q(lb[:,3])}  stop=own-prev {lb[:,4].mean():.2f}")
