@@ -69,10 +69,6 @@ template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
 #ifndef SAM_EARLY_RELOAD
 #define SAM_EARLY_RELOAD 0
 #endif
-// SAM_LB_EARLY: start a super-tile's carry fold before its own aggregate is complete
-#ifndef SAM_LB_EARLY
-#define SAM_LB_EARLY 0
-#endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
 #endif
@@ -90,7 +86,8 @@ template <typename T, int K> struct Lag {
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int NCARRY = 4;                          // carry (look-back) warps, round-robin over tiles
+constexpr int NCARRY = 4;                          // carry (look-back) warps
+constexpr int NCARRY_P1 = NCARRY + 1;
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
 // threads of a CTA: one compute group (or two: local scans + carry applications) + service warps
@@ -138,7 +135,8 @@ struct Params {
     T bw[K];              // b_d(Uw)
     T bu[K];              // b_d(U)        (one tile)
     T bus[K];             // b_d(M*U)      (one super-tile)
-    T bwin[K];            // b_d(Wn*V*M*U) (one look-back round trip further)
+    T bwinj[NCARRY_P1][K]; // b_d(j*Wn*V*M*U), j <= NCARRY (look-back windows further)
+    int coop;             // all carry warps fold each super-tile's windows together
     T bwn[K];             // b_d(Wn*M*U)   (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bq[8][K];           // b_d(q*Uw),     q < c
@@ -328,7 +326,8 @@ struct Smem {
     static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
     static constexpr int HOB = 16 + MAXS * K * (int)sizeof(T);           // hand-off entry: i32 r, pad, [MAXS][K]
     static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
-    static constexpr int OFF_EQ = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;  // [ELAG][TILE_THREADS][K]
+    static constexpr int OFF_PART = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;   // [2][NCARRY][MAXS][K]
+    static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(T);  // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
 };
 
@@ -651,22 +650,30 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // between CTAs, hence no serial latency).
         const int npair = s * c;
         const int cw = warp - (NCW + 2);
-        for (int r = cw;; r += NCARRY) {  // this CTA's r-th super-tile
+        // p.coop: the fold needs several windows (large states, tuples): all carry warps work on
+        // every super-tile, warp w folding windows w, w+NCARRY, ... (round trips in parallel);
+        // otherwise the carry warps take super-tiles round-robin, one warp folding all windows
+        const bool coop = p.coop != 0;
+        const bool lead = !coop || cw == 0;  // finishes the super-tile (hand-off, sub-tile states)
+        const int WV = p.Wn * V;             // super-tiles per window
+        T* const part_s = (T*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
+        for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
             const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
             if ((uint64_t)tile >= p.num_super) break;
             const int64_t Sprev = r == 0 ? (int64_t)-1 : tile - gridDim.x;
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
-#if !SAM_LB_EARLY
-            // Wait for this warp's barrier: the aggregator arrives on it when super-tile r is fully
-            // aggregated, and only after this warp took super-tile r - NCARRY (cw_taken), so the
-            // barrier is never more than one phase ahead and the parity below is unambiguous.
-            mbar_wait(&bar_cw[cw], (uint32_t)((r / NCARRY) & 1));
-            __syncwarp();
-            if (lane == 0) cw_taken[cw] = r;
-#endif
-            if (lane == 0) SAM_TRACE(4, tile * p.M);
+            const int bw = coop ? (int)(r % NCARRY) : cw;  // the aggregator's barrier for super-tile r
+            if (lead) {
+                // Wait for the aggregator: it arrives on bar_cw[r % NCARRY] when super-tile r is
+                // fully aggregated, and only after super-tile r - NCARRY was taken (cw_taken), so the
+                // barrier is never more than one phase ahead and the parity below is unambiguous.
+                mbar_wait(&bar_cw[bw], (uint32_t)((r / NCARRY) & 1));
+                __syncwarp();
+                if (lane == 0) cw_taken[bw] = r;
+            }
+            if (lane == 0 && lead) SAM_TRACE(4, tile * p.M);
 
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, T* out) {
@@ -685,19 +692,20 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 
             T C[K];
             {
-                // lane = (jl, mlb); window row vv holds the super-tile at distance d = jl + Wn*vv
-                // before basei; rows beyond Sprev hold nothing, the row AT Sprev holds this CTA's
-                // previous inclusive state (or, for r = 0, the seed of virtual super-tile -1)
+                // lane = (jl, mlb); row vv of window j holds the super-tile at distance
+                // d = j*WV + jl + Wn*vv before S-1; rows beyond Sprev hold nothing, the row AT Sprev
+                // holds this CTA's previous inclusive state (or, for r = 0, the seed of super-tile -1)
                 const int Wn = p.Wn;
                 const int jl = lane / s, mlb = lane - jl * s;
                 const bool active = jl < Wn;
                 T total[K], Pm[K];
+                const int j0 = coop ? cw : 0, jstep = coop ? NCARRY : 1;
 #pragma unroll
-                for (int t = 0; t < K; ++t) { total[t] = T(0); Pm[t] = (t == 0) ? T(1) : T(0); }
-                int64_t basei = tile - 1;
-                bool first = true;
+                for (int t = 0; t < K; ++t) { total[t] = T(0); Pm[t] = p.bwinj[j0][t]; }  // Pm = M(j0 WV US)
                 int npoll = 0;
-                for (;;) {
+                for (int j = j0;; j += jstep) {
+                    const int64_t basei = tile - 1 - (int64_t)j * WV;
+                    if (basei < Sprev) break;  // window j starts beyond Sprev: nothing left for this warp
                     unsigned long long w[V][K][W1];
                     int st[V];  // 0 pending, 1 aggregate valid, 2 previous inclusive / seed, 3 nothing
 #pragma unroll
@@ -706,7 +714,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         st[vv] = !active ? 3 : (idx > Sprev ? 0 : (idx == Sprev ? 2 : 3));
                     }
                     for (;;) {
-                        if (p.trace && lane == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
+                        if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
                         bool pend = false;
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
@@ -729,11 +737,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                 pend |= !ok;
                             }
                         }
-                        if (p.trace && lane == 0 && npoll == 0) SAM_TRACE(9, tile * p.M);
+                        if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(9, tile * p.M);
                         ++npoll;
                         if (!__any_sync(0xffffffffu, pend)) break;
                     }
-                    const bool last = basei - (int64_t)Wn * V < Sprev;  // this window holds Sprev
+                    const bool last = basei - (int64_t)WV < Sprev;  // this window holds Sprev
                     if (p.trace && lane == 0 && last) {
                         SAM_TRACE(10, tile * p.M);
                         p.trace[(size_t)(tile * p.M) * 16 + 11] = npoll;
@@ -743,7 +751,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         while (*rt != r - 1) __nanosleep(20);
                         __syncwarp();
                     }
-                    // fold.  This lane's rows sit at d = jl + Wn*vv, so by Horner in vv:
+                    // fold.  This lane's rows sit at d = jl + Wn*vv (+ j*WV), so by Horner in vv:
                     //   sum_vv M((jl + Wn vv) US) X_vv = M(jl US) (X_0 + M(Wn US)(X_1 + M(Wn US)(X_2 + ...)))
                     T Y[K];
 #pragma unroll
@@ -779,7 +787,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn US) Y + X
                                 T acc2 = Y[t] + X[t];
 #pragma unroll
-                                for (int j = 0; j < t; ++j) acc2 += p.bwn[t - j] * Y[j];
+                                for (int jj = 0; jj < t; ++jj) acc2 += p.bwn[t - jj] * Y[jj];
                                 Y[t] = acc2;
                             }
                         }
@@ -789,7 +797,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int t = K - 1; t >= 1; --t) {
                             T acc2 = Y[t];
 #pragma unroll
-                            for (int j = 0; j < t; ++j) acc2 += bl_s[jl * K + (t - j)] * Y[j];
+                            for (int jj = 0; jj < t; ++jj) acc2 += bl_s[jl * K + (t - jj)] * Y[jj];
                             Y[t] = acc2;
                         }
                     }
@@ -800,44 +808,48 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             if (jl + off < Wn) Y[t] += o;
                         }
                     }
-                    // lanes jl == 0 hold this window's sum; total += M(offset) Y
-                    if (first) {
+                    // lanes jl == 0 hold this window's sum; total += M(j WV US) Y
 #pragma unroll
-                        for (int t = 0; t < K; ++t) total[t] = Y[t];
-                    } else {
+                    for (int t = K - 1; t >= 0; --t) {
+                        T acc2 = Y[t];
 #pragma unroll
-                        for (int t = 0; t < K; ++t) {
-                            T acc2 = Y[t];
-#pragma unroll
-                            for (int j = 0; j < t; ++j) acc2 += Pm[t - j] * Y[j];
-                            total[t] += acc2;
-                        }
+                        for (int jj = 0; jj < t; ++jj) acc2 += Pm[t - jj] * Y[jj];
+                        total[t] += acc2;
                     }
                     if (last) break;
-                    {   // Pm <- Pm * M(Wn*V*US)  (truncated polynomial product)
+                    {   // Pm <- Pm * M(jstep*WV*US)  (truncated polynomial product)
                         T np[K];
 #pragma unroll
                         for (int d = 0; d < K; ++d) {
                             T acc2 = T(0);
 #pragma unroll
-                            for (int e2 = 0; e2 <= d; ++e2) acc2 += Pm[e2] * p.bwin[d - e2];
+                            for (int e2 = 0; e2 <= d; ++e2) acc2 += Pm[e2] * p.bwinj[jstep][d - e2];
                             np[d] = acc2;
                         }
 #pragma unroll
                         for (int d = 0; d < K; ++d) Pm[d] = np[d];
                     }
-                    basei -= (int64_t)Wn * V;
-                    first = false;
+                }
+                if (coop) {  // sum the warps' partial folds (all already at their absolute offsets)
+                    T* slot = part_s + ((r & 1) * NCARRY + cw) * MAXS * K;
+                    if (lane_ok) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) slot[lane * K + t] = total[t];
+                    }
+                    named_bar_sync(4, NCARRY * 32);
+                    if (lead && lane_ok) {
+                        for (int w2 = 1; w2 < NCARRY; ++w2) {
+                            const T* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
+#pragma unroll
+                            for (int t = 0; t < K; ++t) total[t] += o[lane * K + t];
+                        }
+                    }
                 }
 #pragma unroll
                 for (int t = 0; t < K; ++t) C[t] = total[t];
             }
+            if (!lead) continue;
 
-#if SAM_LB_EARLY
-            mbar_wait(&bar_cw[cw], (uint32_t)((r / NCARRY) & 1));
-            __syncwarp();
-            if (lane == 0) cw_taken[cw] = r;
-#endif
             const int cnt = sub_of[2 * (i0 % NQ) + 1];
             const int il = i0 + cnt - 1;                 // its last iteration
             const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate

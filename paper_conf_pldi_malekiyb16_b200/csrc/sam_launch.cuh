@@ -75,6 +75,13 @@ struct KernelInfo {
     std::mutex mu;
 };
 
+// persistent grid: all co-resident CTAs, at most one per super-tile
+inline uint64_t grid_of(int blocks_per_sm, int num_sms, uint64_t num_super) {
+    uint64_t grid = (uint64_t)blocks_per_sm * (uint64_t)num_sms;
+    if (grid > num_super) grid = num_super;
+    return grid < 1 ? 1 : grid;
+}
+
 template <typename T, int K>
 cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     using S = Smem<T, K>;
@@ -146,7 +153,7 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     mcol<T>(geo.U, K, p.bu);
     mcol<T>(US, K, p.bus);
     constexpr int V = LB<T, K>::V;
-    mcol<T>((int64_t)geo.Wn * V * US, K, p.bwin);
+    for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * V * US, K, p.bwinj[j]);
     mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];
@@ -160,11 +167,17 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, p.bkw[l]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
+    // carry warps cooperate on each super-tile when its fold spans 3 or more windows
+    {
+        const uint64_t wv = (uint64_t)geo.Wn * V;
+        const uint64_t P = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
+        p.coop = 1;  // measured faster for every config tried, also single-window folds
+        (void)P; (void)wv;
+        if (const char* env = getenv("SAM_COOP")) p.coop = atoi(env) != 0;  // experiments
+    }
     // Static schedule (CTA b owns super-tiles b, b+P, ...): every CTA waits on aggregates of the
     // others, so all P CTAs must be co-resident -- a cooperative launch guarantees it (or fails).
-    uint64_t grid = (uint64_t)info.max_blocks_per_sm * (uint64_t)a.num_sms;
-    if (grid > p.num_super) grid = p.num_super;
-    if (grid < 1) grid = 1;
+    const uint64_t grid = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
     cudaLaunchConfig_t cfg;
     memset(&cfg, 0, sizeof(cfg));
     cfg.gridDim = dim3((unsigned)grid);
