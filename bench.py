@@ -109,8 +109,10 @@ class ClockSampler:
                 if val.lower().startswith("active"):
                     reasons.add(name)
         loaded = [x for x, w in zip(sm, watts) if w > 250] or sm
+        lw = [w for w in watts if w > 250] or watts
         return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sm), "samples_under_load": len(loaded)}
+                "reasons": sorted(reasons), "samples": len(sm), "samples_under_load": len(loaded),
+                "power_w": statistics.median(lw) if lw else None}
 
 
 def dist_env():

@@ -42,6 +42,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <string.h>
+
 #include <type_traits>
 
 #include "sam_algebra.h"
@@ -56,6 +58,48 @@ template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 27; };
 template <> struct Cfg<float>    { static constexpr int ITEMS = 27; };
 template <> struct Cfg<uint64_t> { static constexpr int ITEMS = 13; };
 template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
+// VEC (tuple 1, 16-B aligned input): a thread's items are contiguous and 16-B aligned, read and
+// written with 128-bit shared-memory accesses (ITEMS*sizeof(T) = 112 B: the 8 addresses of a
+// quarter-warp phase fall in distinct 16-B bank groups, conflict free)
+template <typename T, bool VEC> struct Items {
+    static constexpr int V = VEC ? 112 / (int)sizeof(T) : Cfg<T>::ITEMS;
+};
+// 128-bit shared-memory load / store of N consecutive elements (16-B aligned)
+template <typename T, int N>
+__device__ __forceinline__ void lds_vec(const T* p, T (&d)[N]) {
+    constexpr int E = 16 / (int)sizeof(T);
+    if constexpr (N % E != 0) {  // not vectorisable (never taken at run time: VEC kernels only)
+#pragma unroll
+        for (int i = 0; i < N; ++i) d[i] = p[i];
+        return;
+    }
+#pragma unroll
+    for (int q = 0; q < N / E; ++q) {
+        const uint4 v = reinterpret_cast<const uint4*>(p)[q];
+        T t[E];
+        memcpy(t, &v, 16);
+#pragma unroll
+        for (int j = 0; j < E; ++j) d[q * E + j] = t[j];
+    }
+}
+template <typename T, int N>
+__device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
+    constexpr int E = 16 / (int)sizeof(T);
+    if constexpr (N % E != 0) {
+#pragma unroll
+        for (int i = 0; i < N; ++i) p[i] = d[i];
+        return;
+    }
+#pragma unroll
+    for (int q = 0; q < N / E; ++q) {
+        T t[E];
+#pragma unroll
+        for (int j = 0; j < E; ++j) t[j] = d[q * E + j];
+        uint4 v;
+        memcpy(&v, t, 16);
+        reinterpret_cast<uint4*>(p)[q] = v;
+    }
+}
 // Pipeline shape by per-thread state size K * sizeof(T):
 //   <= 8 B : 3 local-scan buffers, 3 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
 //   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
@@ -69,14 +113,28 @@ template <> struct Cfg<double>   { static constexpr int ITEMS = 13; };
 #ifndef SAM_EARLY_RELOAD
 #define SAM_EARLY_RELOAD 0
 #endif
+// back-off (ns) of the look-back re-polls, of idle compute warps and of the idle producer
+#ifndef SAM_POLL_NS
+#define SAM_POLL_NS 0
+#endif
+#ifndef SAM_IDLE_NS
+#define SAM_IDLE_NS 32
+#endif
+#ifndef SAM_PROD_NS
+#define SAM_PROD_NS 16
+#endif
+#ifndef SAM_LAG8
+#define SAM_LAG8 12
+#endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
 #endif
 template <typename T, int K> struct Lag {
     static constexpr int SB = K * (int)sizeof(T);
     static constexpr bool SMEM = SB <= 16;           // pending local states in shared memory
-    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? 12 : (SB <= 16 ? 8 : 4));
-    static constexpr int MMAX = SB <= 8 ? 4 : 2;     // max tiles per super-tile (look-back unit)
+    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : 4));
+    // max tiles per super-tile (look-back unit); measured: 3 for 4-byte, 2 for 8-byte elements
+    static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : 2;
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
     static constexpr int NB2 = SB <= 8 ? 4 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
@@ -296,11 +354,11 @@ template <> struct IsInt<uint64_t> { static constexpr bool value = true; };
 // ------------------------------------------------------------------------------------------
 // shared-memory layout
 // ------------------------------------------------------------------------------------------
-template <typename T, int K>
-struct Smem {
-    static constexpr int ITEMS = Cfg<T>::ITEMS;
+template <typename T, int K, bool VEC, int NB2_>
+struct SmemL {
+    static constexpr int ITEMS = Items<T, VEC>::V;
     static constexpr int NB1 = Lag<T, K>::NB1;
-    static constexpr int NB2 = Lag<T, K>::NB2;
+    static constexpr int NB2 = NB2_;
     static constexpr int LAG = Lag<T, K>::LAG;
     static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
     static constexpr int ELAG = Lag<T, K>::SMEM ? LAG : 0;          // smem-resident pending states
@@ -330,14 +388,18 @@ struct Smem {
     static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(T);  // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
 };
+// one carry-application buffer fewer when the larger VEC tiles would not fit
+template <typename T, int K, bool VEC>
+struct Smem : std::conditional_t<(SmemL<T, K, VEC, Lag<T, K>::NB2>::BYTES <= 227 * 1024),
+                                 SmemL<T, K, VEC, Lag<T, K>::NB2>, SmemL<T, K, VEC, Lag<T, K>::NB2 - 1>> {};
 
 // ------------------------------------------------------------------------------------------
 // the kernel
 // ------------------------------------------------------------------------------------------
-template <typename T, int K>
+template <typename T, int K, bool VEC>
 __global__ void __launch_bounds__(Threads<T, K>::VALUE, 1)
 sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
-    using S = Smem<T, K>;
+    using S = Smem<T, K, VEC>;
     constexpr int ITEMS = S::ITEMS;
     constexpr int NB1 = S::NB1;
     constexpr int NB2 = S::NB2;
@@ -348,7 +410,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int W1 = TagW<T>::W;      // tagged words per published value
     constexpr int V = LB<T, K>::V;
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
-    static_assert(ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
+    static_assert(VEC || ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
     static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 4, "ring sizes");
     static_assert(S::BYTES <= 227 * 1024, "shared memory budget");
 
@@ -519,7 +581,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     continue;
                 }
                 if (jend >= 0 && j3 == jend) break;
-                __nanosleep(16);
+                __nanosleep(SAM_PROD_NS);
             }
             bulk_wait_all0();
         }
@@ -740,6 +802,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(9, tile * p.M);
                         ++npoll;
                         if (!__any_sync(0xffffffffu, pend)) break;
+                        if (SAM_POLL_NS > 0) __nanosleep(SAM_POLL_NS);  // back off before re-polling L2
                     }
                     const bool last = basei - (int64_t)WV < Sprev;  // this window holds Sprev
                     if (p.trace && lane == 0 && last) {
@@ -988,6 +1051,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     // all ITEMS loads first: interleaving them with the (possibly aliasing, as far
                     // as the compiler knows) stores would serialise every item on an smem round trip
                     T xv[ITEMS];
+                    if constexpr (VEC && !SLOW) {
+                        lds_vec<T, ITEMS>(xs + base_loc, xv);
+                    } else {
 #pragma unroll
                     for (int i = 0; i < ITEMS; ++i) {
                         const int el = base_loc + i * s;
@@ -999,6 +1065,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             xv[i] = xs[el];
                         }
                     }
+                    }
+                    T ov[VEC && !SLOW ? ITEMS : 1];
 #pragma unroll
                     for (int i = 0; i < ITEMS; ++i) {
                         const int el = base_loc + i * s;
@@ -1029,10 +1097,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                                 for (int t = 0; t < K; ++t) p.final_state[m * K + t] = y[t];
                             }
+                        } else if constexpr (VEC) {
+                            ov[i] = outv;
                         } else {
                             xs[el] = outv;
                         }
                     }
+                    if constexpr (VEC && !SLOW) sts_vec<T, ITEMS>(xs + base_loc, ov);
                 };
                 using TT = std::true_type;
                 using FF = std::false_type;
@@ -1065,7 +1136,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             T acc[K];
 #pragma unroll
             for (int t = 0; t < K; ++t) acc[t] = T(0);
-            if (!masked) {
+            if (VEC && !masked) {
+                T xv[ITEMS];
+                lds_vec<T, ITEMS>(xs + base_loc, xv);
+#pragma unroll
+                for (int it = 0; it < ITEMS; ++it) {
+                    acc[0] += xv[it];
+#pragma unroll
+                    for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                }
+            } else if (!masked) {
 #pragma unroll
                 for (int it = 0; it < ITEMS; ++it) {
                     const T x = xs[base_loc + it * s];
@@ -1235,7 +1315,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 } else if (end >= 0 && p1_next >= end) {
                     break;
                 }
-                __nanosleep(32);  // nothing ready: yield issue slots to the other warps
+                __nanosleep(SAM_IDLE_NS);  // nothing ready: yield issue slots to the other warps
             }
         }
     }

@@ -68,7 +68,7 @@ struct LaunchArgs {
 template <typename T>
 inline int items_of() { return Cfg<T>::ITEMS; }
 
-template <typename T, int K>
+template <typename T, int K, bool VEC>
 struct KernelInfo {
     int max_blocks_per_sm = 0;
     bool ready = false;
@@ -82,24 +82,25 @@ inline uint64_t grid_of(int blocks_per_sm, int num_sms, uint64_t num_super) {
     return grid < 1 ? 1 : grid;
 }
 
-template <typename T, int K>
-cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
-    using S = Smem<T, K>;
-    static KernelInfo<T, K> info;
+template <typename T, int K, bool VEC>
+cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
+    using S = Smem<T, K, VEC>;
+    constexpr int ITEMS = Items<T, VEC>::V;
+    static KernelInfo<T, K, VEC> info;
     {
         std::lock_guard<std::mutex> lk(info.mu);
         if (!info.ready) {
-            cudaError_t e = cudaFuncSetAttribute(sam_scan_kernel<T, K>,
+            cudaError_t e = cudaFuncSetAttribute(sam_scan_kernel<T, K, VEC>,
                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES);
             if (e != cudaSuccess) return e;
             int nb = 0;
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K>, Threads<T, K>::VALUE, S::BYTES);
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K, VEC>, Threads<T, K>::VALUE, S::BYTES);
             if (e != cudaSuccess) return e;
             info.max_blocks_per_sm = nb > 0 ? nb : 1;
             info.ready = true;
         }
     }
-    const Geom geo = make_geom(a.s, Cfg<T>::ITEMS);
+    const Geom geo = make_geom(a.s, ITEMS);
     Params<T, K> p;
     memset(&p, 0, sizeof(p));
     p.in = (const T*)a.in;
@@ -148,7 +149,7 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
         p.num_super = (p.num_tiles + m - 1) / m;
     }
     const int64_t US = (int64_t)p.M * geo.U;  // lane length of a super-tile
-    mcol<T>(Cfg<T>::ITEMS, K, p.bc);
+    mcol<T>(ITEMS, K, p.bc);
     mcol<T>(geo.Uw, K, p.bw);
     mcol<T>(geo.U, K, p.bu);
     mcol<T>(US, K, p.bus);
@@ -157,13 +158,13 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];
-        mcol<T>((int64_t)v * Cfg<T>::ITEMS, K, b);
+        mcol<T>((int64_t)v * ITEMS, K, b);
         for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
     }
     for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
     for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, p.bl[j]);
     for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, p.bsub[j]);
-    for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * Cfg<T>::ITEMS, K, p.bks[l]);
+    for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * ITEMS, K, p.bks[l]);
     for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, p.bkw[l]);
 
     // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
@@ -189,9 +190,16 @@ cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, sam_scan_kernel<T, K>, p);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, sam_scan_kernel<T, K, VEC>, p);
     if (launches && e == cudaSuccess) ++*launches;
     return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+// tuple 1 with a 16-B aligned input: the 128-bit shared-memory variant
+template <typename T, int K>
+cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
+    const bool vec = a.s == 1 && ((uintptr_t)a.in & 15) == 0 && getenv("SAM_NO_VEC") == nullptr;
+    return vec ? launch_scan_impl<T, K, true>(a, launches) : launch_scan_impl<T, K, false>(a, launches);
 }
 
 template <typename T>
