@@ -129,10 +129,18 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
 #endif
+// states of 17..32 B (int32 orders 5-8, int64 orders 3-4): pending in shared memory, LAG 6
+#ifndef SAM_SMEM32
+#define SAM_SMEM32 1
+#endif
+#ifndef SAM_LAG32
+#define SAM_LAG32 6
+#endif
 template <typename T, int K> struct Lag {
     static constexpr int SB = K * (int)sizeof(T);
-    static constexpr bool SMEM = SB <= 16;           // pending local states in shared memory
-    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : 4));
+    static constexpr bool BIG32 = SAM_SMEM32 && SB > 16 && SB <= 32;
+    static constexpr bool SMEM = SB <= 16 || BIG32;  // pending local states in shared memory
+    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : (BIG32 ? SAM_LAG32 : 4)));
     // max tiles per super-tile (look-back unit); measured: 3 for 4-byte, 2 for 8-byte elements
     static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : 2;
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
@@ -140,7 +148,7 @@ template <typename T, int K> struct Lag {
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = SMEM && K >= SAM_SPLIT_MIN_K;
+    static constexpr bool SPLIT = SMEM && !BIG32 && K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
