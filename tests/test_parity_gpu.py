@@ -1,8 +1,9 @@
 """GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
 
 Integers bit-exact; floats within rtol*sqrt(n*k)*A (R7) plus exact checks on
-integer-valued inputs.  Sizes span several tiles (T = 2400..3840 elements) and a ragged tail; the
-look-back sizes span more tiles than a look-back window (32/s tiles).
+integer-valued inputs.  Sizes span several tiles (T = 3328..7168 elements) and a ragged tail; the
+multi-round sizes give every CTA several super-tiles, so the carry schedule's hand-off of a CTA's
+own inclusive state and its multi-window folds of the P-1 aggregates in between are exercised.
 """
 from __future__ import annotations
 
@@ -197,3 +198,24 @@ def test_scan_host_pipeline(name):
     for k, s in ((1, 1), (3, 4)):
         y = S.scan_host(x, k, s, True)
         compare(name, xn, y.numpy(), k, s, True)
+
+
+@pytest.mark.parametrize("name,k,s", [("i32", 1, 1), ("i32", 2, 1), ("i32", 3, 1), ("i64", 1, 1), ("i64", 4, 1),
+                                      ("i64", 1, 3), ("i64", 2, 8), ("i32", 8, 1), ("i64", 8, 5)])
+def test_multi_round_schedule(name, k, s):
+    # > 3 super-tiles per CTA on 148 SMs (tiles of 3328..7168 elements, super-tiles of 2-3 tiles)
+    n = 148 * 3 * 7168 * 3 + 4099
+    x = synth.make(n, name, "uniform", seed=synth.SEED_BASE + 4242 + 16 * k + s)
+    for inclusive in (True, False):
+        compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
+
+
+@pytest.mark.parametrize("name,k,s", [("f32", 1, 1), ("f64", 1, 1), ("f32", 2, 3), ("f64", 4, 4)])
+def test_float_bit_deterministic(name, k, s):
+    # fixed association order (static carry schedule): identical bits run to run (R6)
+    S = sam()
+    x = torch.from_numpy(synth.make(1 << 24, name, "unif01", seed=synth.SEED_BASE + 99 + k + s)).cuda()
+    y0 = S.scan(x, order=k, tuple=s, inclusive=True)
+    for _ in range(3):
+        y1 = S.scan(x, order=k, tuple=s, inclusive=True)
+        assert torch.equal(y0.view(torch.uint8), y1.view(torch.uint8))
