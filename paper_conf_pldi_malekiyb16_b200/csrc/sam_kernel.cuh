@@ -1075,6 +1075,36 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                     }
                     T ov[VEC && !SLOW ? ITEMS : 1];
+                    if constexpr (VEC && !SLOW && K == 1) {
+                        // order 1: chunked prefix (ITEMS/7 independent chains of 7, then chunk offsets):
+                        // dependent-add depth 7 + ITEMS/7 instead of ITEMS
+                        constexpr int L = 7, CH = ITEMS / L;
+                        T pre[ITEMS];
+#pragma unroll
+                        for (int c2 = 0; c2 < CH; ++c2) {
+                            pre[c2 * L] = xv[c2 * L];
+#pragma unroll
+                            for (int j = 1; j < L; ++j) pre[c2 * L + j] = pre[c2 * L + j - 1] + xv[c2 * L + j];
+                        }
+                        T off = y[0];
+#pragma unroll
+                        for (int c2 = 0; c2 < CH; ++c2) {
+                            const T base = off;
+                            off += pre[c2 * L + L - 1];
+#pragma unroll
+                            for (int j = 0; j < L; ++j) pre[c2 * L + j] += base;
+                        }
+                        if constexpr (EXCL) {
+                            ov[0] = ring[0];  // y at the position before the thread's first item
+#pragma unroll
+                            for (int i = 1; i < ITEMS; ++i) ov[i] = pre[i - 1];
+                        } else {
+#pragma unroll
+                            for (int i = 0; i < ITEMS; ++i) ov[i] = pre[i];
+                        }
+                        sts_vec<T, ITEMS>(xs + base_loc, ov);
+                        return;
+                    }
 #pragma unroll
                     for (int i = 0; i < ITEMS; ++i) {
                         const int el = base_loc + i * s;
@@ -1147,11 +1177,18 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if (VEC && !masked) {
                 T xv[ITEMS];
                 lds_vec<T, ITEMS>(xs + base_loc, xv);
+                if constexpr (K == 1) {  // order 1 needs only the sum: 4 independent chains
+                    T a4[4] = {T(0), T(0), T(0), T(0)};
+#pragma unroll
+                    for (int it = 0; it < ITEMS; ++it) a4[it & 3] += xv[it];
+                    acc[0] = (a4[0] + a4[1]) + (a4[2] + a4[3]);
+                } else {
 #pragma unroll
                 for (int it = 0; it < ITEMS; ++it) {
                     acc[0] += xv[it];
 #pragma unroll
                     for (int t = 1; t < K; ++t) acc[t] += acc[t - 1];
+                }
                 }
             } else if (!masked) {
 #pragma unroll

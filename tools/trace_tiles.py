@@ -6,8 +6,13 @@ import paper_conf_pldi_malekiyb16_b200 as S
 dt, logn, k, s = sys.argv[1], int(sys.argv[2]), int(sys.argv[3]), int(sys.argv[4])
 n = 1 << logn
 x = synth.make_torch(n, dt, "uniform", device="cuda"); y = torch.empty_like(x)
-for _ in range(3): S.scan(x, k, s, True, out=y)
-torch.cuda.synchronize()
+import time
+soak = float(os.environ.get("SOAK_S", "0"))  # sustained-load clocks (power cap) before the traced launch
+t0 = time.time()
+while True:
+    for _ in range(3): S.scan(x, k, s, True, out=y)
+    torch.cuda.synchronize()
+    if time.time() - t0 >= soak: break
 tr = torch.zeros(16 * (n // 1000 + 16), dtype=torch.int64, device="cuda")
 S.lib().sam_debug_set_trace(ctypes.c_void_p(tr.data_ptr()))
 S.scan(x, k, s, True, out=y); torch.cuda.synchronize()
