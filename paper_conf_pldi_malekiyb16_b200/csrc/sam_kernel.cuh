@@ -203,6 +203,7 @@ struct Params {
     T bus[K];             // b_d(M*U)      (one super-tile)
     T bwinj[NCARRY_P1][K]; // b_d(j*Wn*V*M*U), j <= NCARRY (look-back windows further)
     int coop;             // all carry warps fold each super-tile's windows together
+    int Vr;               // window rows used per round trip (<= V)
     T bwn[K];             // b_d(Wn*M*U)   (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bq[8][K];           // b_d(q*Uw),     q < c
@@ -725,7 +726,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // otherwise the carry warps take super-tiles round-robin, one warp folding all windows
         const bool coop = p.coop != 0;
         const bool lead = !coop || cw == 0;  // finishes the super-tile (hand-off, sub-tile states)
-        const int WV = p.Wn * V;             // super-tiles per window
+        const int WV = p.Wn * p.Vr;          // super-tiles per window
         T* const part_s = (T*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
         for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
@@ -781,7 +782,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                     for (int vv = 0; vv < V; ++vv) {
                         const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                        st[vv] = !active ? 3 : (idx > Sprev ? 0 : (idx == Sprev ? 2 : 3));
+                        st[vv] = (!active || vv >= p.Vr) ? 3 : (idx > Sprev ? 0 : (idx == Sprev ? 2 : 3));
                     }
                     for (;;) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
@@ -908,6 +909,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int t = 0; t < K; ++t) slot[lane * K + t] = total[t];
                     }
                     named_bar_sync(4, NCARRY * 32);
+                    if (lead && lane == 0) SAM_TRACE(13, tile * p.M);
                     if (lead && lane_ok) {
                         for (int w2 = 1; w2 < NCARRY; ++w2) {
                             const T* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
@@ -948,6 +950,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     *(volatile int*)ho = r;
                 }
             }
+            if (lane == 0) SAM_TRACE(14, tile * p.M);
             // each sub-tile j: C_j = M(j U) C + P_j, then per-warp incoming states
             // C_{m,q} = M(q*Uw) C_{j,m} + E_{m,q}  (E in wq, from the combine)
             for (int j = 0; j < cnt; ++j) {

@@ -136,7 +136,11 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
     {
         uint64_t m = p.num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
         if (m < 1) m = 1;
-        if (m > (uint64_t)Lag<T, K>::MMAX) m = Lag<T, K>::MMAX;
+        // measured: tuple 1: 3 (4-byte) / 2 (8-byte) tiles; tuples (more carry-team work per unit):
+        // 3, or 4 for >= 16-B states
+        const int SB = K * (int)sizeof(T);
+        const uint64_t mmax = a.s == 1 ? (uint64_t)Lag<T, K>::MMAX : (SB >= 16 ? 4u : 3u);
+        if (m > mmax) m = mmax;
         if (const char* env = getenv("SAM_SUPER_TILE")) {  // experiments: force a smaller super-tile
             const int f = atoi(env);
             if (f >= 1 && f <= 8) m = (uint64_t)f;
@@ -154,7 +158,17 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
     mcol<T>(geo.U, K, p.bu);
     mcol<T>(US, K, p.bus);
     constexpr int V = LB<T, K>::V;
-    for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * V * US, K, p.bwinj[j]);
+    {   // window rows: enough for the carry warps together to cover the P-1 aggregates in one round trip
+        const uint64_t P = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
+        const uint64_t rows = (P + geo.Wn - 1) / geo.Wn;
+        uint64_t vr = (rows + NCARRY - 1) / NCARRY;
+        if (vr < 1) vr = 1;
+        if (vr > (uint64_t)V) vr = V;
+        vr = V;  // measured: the full register budget per round trip beats spreading rows over warps
+        if (const char* env = getenv("SAM_VR")) { const int f = atoi(env); if (f >= 1 && f <= V) vr = f; }
+        p.Vr = (int)vr;
+    }
+    for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * p.Vr * US, K, p.bwinj[j]);
     mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];

@@ -19,11 +19,20 @@ S.scan(x, k, s, True, out=y); torch.cuda.synchronize()
 S.lib().sam_debug_set_trace(None)
 t = tr.cpu().numpy().reshape(-1, 16)
 t = t[t[:, 0] > 0]
-extra = t[:, 8:].copy()
-t = t[:, :8] - t[:, 0].min()
+t0 = t[:, 0].min()
+ts_cols = [0, 1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 13, 14]  # timestamp events (11, 12: counters)
+tf = np.full(t.shape, np.nan)
+for c in range(16):
+    nz = t[:, c] != 0
+    tf[nz, c] = (t[nz, c] - t0).astype(np.float64) if c in ts_cols else t[nz, c]
+extra = tf[:, 8:].copy()
+extra[np.isnan(extra)] = 0
+t = tf[:, :8]  # ns since the first claim; NaN = event not recorded for this tile
 names = ["claim", "p1start", "p1done", "aggpub", "lbstart", "inclpub", "p2start", "stored"]
-print(f"{dt} 2^{logn} k={k} s={s}: tiles {len(t)}  span {t.max()/1e3:.1f} us  rate {len(t)/(t.max()/1e3):.1f} tiles/us")
-def q(a): return " ".join(f"{np.percentile(a, pp):7.2f}" for pp in (10, 50, 90, 99))
+print(f"{dt} 2^{logn} k={k} s={s}: tiles {len(t)}  span {np.nanmax(t)/1e3:.1f} us  rate {len(t)/(np.nanmax(t)/1e3):.1f} tiles/us")
+def q(a):
+    a = np.asarray(a, dtype=np.float64); a = a[~np.isnan(a)]
+    return " ".join(f"{np.percentile(a, pp):7.2f}" for pp in (10, 50, 90, 99)) if a.size else "n/a"
 print("interval (us)            p10     p50     p90     p99")
 for a_, b_ in [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5), (5, 6), (6, 7), (0, 3), (3, 5), (0, 7)]:
     d = (t[:, b_] - t[:, a_]) / 1e3
@@ -39,6 +48,17 @@ ev = ev[np.argsort(ev[:, 0], kind="stable")]
 occ = np.cumsum(ev[:, 1])
 print(f"parked tiles: p50 {np.percentile(occ, 50):.0f}  p90 {np.percentile(occ, 90):.0f}  max {occ.max():.0f}"
       f"  (~{np.percentile(occ, 50) * tile_bytes / 2**20:.1f} / {occ.max() * tile_bytes / 2**20:.1f} MiB)")
-lb = extra[extra[:, 0] > 0]
+lb = extra[extra[:, 0] != 0]
 if len(lb):
     print(f"look-back units {len(lb)}: first poll RTT {q((lb[:,1]-lb[:,0])/1e3)}  loop {q((lb[:,2]-lb[:,0])/1e3)}  polls {q(lb[:,3])}  stop=own-prev {lb[:,4].mean():.2f}")
+# super-tile view: aggregate of its last sub-tile -> carry team starts -> first sub-tile's carry ready
+first = np.nonzero(~np.isnan(t[:, 4]))[0]
+if len(first) > 2:
+    M = int(np.median(np.diff(first)))
+    f = first[first + M - 1 < len(t)]
+    last = f + M - 1
+    us = lambda a: np.asarray(a) / 1e3
+    print(f"super-tiles (M={M}):  lastagg->lbstart {q(us(t[f, 4] - t[last, 3]))}   lbstart->incl {q(us(t[f, 5] - t[f, 4]))}")
+    e = tf[f]
+    print(f"  lbstart->poll0 {q(us(e[:, 8] - e[:, 4]))}  poll0->lbdone {q(us(e[:, 10] - e[:, 8]))}  lbdone->barrier {q(us(e[:, 13] - e[:, 10]))}"
+          f"  barrier->handoff {q(us(e[:, 14] - e[:, 13]))}  handoff->incl0 {q(us(e[:, 5] - e[:, 14]))}")
