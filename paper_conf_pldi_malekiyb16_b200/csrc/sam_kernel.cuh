@@ -204,6 +204,7 @@ struct Params {
     T bwinj[NCARRY_P1][K]; // b_d(j*Wn*V*M*U), j <= NCARRY (look-back windows further)
     int coop;             // all carry warps fold each super-tile's windows together
     int Vr;               // window rows used per round trip (<= V)
+    T bprev[K];           // b_d((P-1)*M*U): from this CTA's previous super-tile to the one before S
     T bwn[K];             // b_d(Wn*M*U)   (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bq[8][K];           // b_d(q*Uw),     q < c
@@ -782,7 +783,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                     for (int vv = 0; vv < V; ++vv) {
                         const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                        st[vv] = (!active || vv >= p.Vr) ? 3 : (idx > Sprev ? 0 : (idx == Sprev ? 2 : 3));
+                        st[vv] = (!active || vv >= p.Vr || idx <= Sprev) ? 3 : 0;
                     }
                     for (;;) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
@@ -818,11 +819,6 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         SAM_TRACE(10, tile * p.M);
                         p.trace[(size_t)(tile * p.M) * 16 + 11] = npoll;
                     }
-                    if (last && Sprev >= 0) {  // previous inclusive state: wait for its hand-off entry
-                        const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
-                        while (*rt != r - 1) __nanosleep(20);
-                        __syncwarp();
-                    }
                     // fold.  This lane's rows sit at d = jl + Wn*vv (+ j*WV), so by Horner in vv:
                     //   sum_vv M((jl + Wn vv) US) X_vv = M(jl US) (X_0 + M(Wn US)(X_1 + M(Wn US)(X_2 + ...)))
                     T Y[K];
@@ -841,14 +837,6 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                 } else {
                                     X[t] = Bits<T>::from((w[vv][t][0] & 0xffffffffull) | (w[vv][t][1] << 32));
                                 }
-                            }
-                        } else if (st[vv] == 2) {
-                            if (Sprev < 0) {
-                                seed_of(mlb, X);
-                            } else {
-                                const T* hv = (const T*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
-#pragma unroll
-                                for (int t = 0; t < K; ++t) X[t] = hv[mlb * K + t];
                             }
                         }
                         if (vv == V - 1) {
@@ -915,6 +903,35 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             const T* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
 #pragma unroll
                             for (int t = 0; t < K; ++t) total[t] += o[lane * K + t];
+                        }
+                    }
+                }
+                if (lead) {
+                    // the CTA's own chain, kept to a few operations: C = F + M((S-1-Sprev) US) I_prev,
+                    // I_prev = this CTA's inclusive state after Sprev (hand-off) or, for r = 0, the seed
+                    // of virtual super-tile -1 (M(S US) computed here, once per CTA)
+                    T pv[K], bcol[K];
+                    bool have = false;
+                    if (Sprev >= 0) {
+                        const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
+                        while (*rt != r - 1) __nanosleep(20);
+                        __syncwarp();
+                        const T* hv = (const T*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
+#pragma unroll
+                        for (int t = 0; t < K; ++t) { pv[t] = hv[ml * K + t]; bcol[t] = p.bprev[t]; }
+                        have = true;
+                    } else if (p.seed) {
+                        seed_of(ml, pv);
+                        mcol<T>(tile * (int64_t)p.M * p.U, K, bcol);
+                        have = true;
+                    }
+                    if (have) {
+#pragma unroll
+                        for (int t = K - 1; t >= 0; --t) {
+                            T acc2 = total[t] + pv[t];
+#pragma unroll
+                            for (int jj = 0; jj < t; ++jj) acc2 += bcol[t - jj] * pv[jj];
+                            total[t] = acc2;
                         }
                     }
                 }

@@ -169,6 +169,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         p.Vr = (int)vr;
     }
     for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * p.Vr * US, K, p.bwinj[j]);
+    mcol<T>((int64_t)(grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super) - 1) * US, K, p.bprev);
     mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
     for (int v = 0; v < 32; ++v) {
         T b[K];
