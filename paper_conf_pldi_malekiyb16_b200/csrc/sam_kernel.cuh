@@ -123,6 +123,10 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_PROD_NS
 #define SAM_PROD_NS 16
 #endif
+// orders >= SAM_KS_MIN_K scan thread/warp k-vector states Kogge-Stone style, lower orders order by order
+#ifndef SAM_KS_MIN_K
+#define SAM_KS_MIN_K 3
+#endif
 #ifndef SAM_LAG8
 #define SAM_LAG8 12
 #endif
@@ -619,7 +623,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
                 T E[K], yl[K];
-                if constexpr (K <= 2) {
+                if constexpr (K < SAM_KS_MIN_K) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) {
                         T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
@@ -1234,7 +1238,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             //   z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]      (5k dependent shuffle stages)
             // Orders >= 3: Kogge-Stone on k-vectors with the carry operator, level l combining
             //   st <- M(2^l ITEMS) st_partner + st                       (5 dependent stages)
-            if constexpr (K <= 2) {
+            if constexpr (K < SAM_KS_MIN_K) {
 #pragma unroll
                 for (int t = 0; t < K; ++t) {
                     T z = acc[t];
