@@ -9,6 +9,6 @@ timeout 300 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/b
 rm -f gpurun_out/bench_configs.jsonl
 for c in C3k8 C3i64k8 C4s8 C5; do timeout 300 python bench.py --config $c --steps 20 --no-e2e --no-cpu >> gpurun_out/bench_configs.jsonl 2>/dev/null; done
 timeout 300 python tools/sweep.py 3 > gpurun_out/sweep.txt 2>&1
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches.csv python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:sam_ -c 20 --csv --log-file gpurun_out/launches.csv python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:sam_scan_kernel -s 8 -c 1 -o gpurun_out/prof_c2 python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
 ls -la gpurun_out
