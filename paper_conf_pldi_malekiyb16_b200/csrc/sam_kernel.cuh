@@ -619,6 +619,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             T* lp = lp_all + qs * S::LA;
 #pragma unroll
             for (int ch = 0; ch < 2; ++ch) {
+                if (32 * ch >= npair) break;  // warp-uniform: second pass only for s = 8
                 const int pair = lane + 32 * ch;
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
@@ -988,6 +989,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
 #pragma unroll
                 for (int ch = 0; ch < 2; ++ch) {
+                    if (32 * ch >= npair) break;  // warp-uniform: second pass only for s = 8
                     const int pair = lane + 32 * ch;
                     const bool ok = pair < npair;
                     const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
