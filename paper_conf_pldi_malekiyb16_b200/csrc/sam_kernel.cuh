@@ -792,23 +792,32 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                     for (;;) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
-                        bool pend = false;
+                        // all loads first, then the tag checks: the loads of a window are then in
+                        // flight together (one round trip), not one after the other
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
                                 const int64_t idx = basei - jl - (int64_t)Wn * vv;
                                 const unsigned long long* src = p.carry + ((size_t)idx * s + mlb) * K * W1;
-                                bool ok = true;
 #pragma unroll
                                 for (int t = 0; t < K; ++t) {
                                     if constexpr (W1 == 1) {
                                         w[vv][t][0] = ld_relaxed_u64(src + t);
-                                        ok &= (uint32_t)(w[vv][t][0] >> 32) == tag;
                                     } else {
                                         ld_relaxed_v2(src + 2 * t, w[vv][t][0], w[vv][t][1]);
-                                        ok &= (uint32_t)(w[vv][t][0] >> 32) == tag &&
-                                              (uint32_t)(w[vv][t][1] >> 32) == tag;
                                     }
+                                }
+                            }
+                        }
+                        bool pend = false;
+#pragma unroll
+                        for (int vv = 0; vv < V; ++vv) {
+                            if (st[vv] == 0) {
+                                bool ok = true;
+#pragma unroll
+                                for (int t = 0; t < K; ++t) {
+                                    ok &= (uint32_t)(w[vv][t][0] >> 32) == tag;
+                                    if constexpr (W1 == 2) ok &= (uint32_t)(w[vv][t][1] >> 32) == tag;
                                 }
                                 st[vv] = ok ? 1 : 0;
                                 pend |= !ok;
