@@ -108,7 +108,8 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_LAG_SMALL
 #define SAM_LAG_SMALL 12
 #endif
-// SAM_EARLY_RELOAD: re-fetch a tile into a carry buffer as soon as its local scan is done (the
+// SAM_EARLY_RELOAD: 1 = re-fetch a tile into a carry buffer as soon as its local scan is done, 2 = as
+// soon as its super-tile's carry fold starts (one L2 round trip before the carry is expected) (the
 // carry application then also waits for the carry) instead of once its carry is known
 #ifndef SAM_EARLY_RELOAD
 #define SAM_EARLY_RELOAD 0
@@ -444,6 +445,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint32_t* sm_tag = (uint32_t*)(smem + S::OFF_TAG);
     volatile int* sm_end = (volatile int*)(smem + S::OFF_TAG + 4);
     volatile int* agg_done = (volatile int*)(smem + S::OFF_TAG + 8);  // iterations aggregated
+    volatile int* lb_started = (volatile int*)(smem + S::OFF_TAG + 20);  // last super-tile whose fold began
     T* wq_all = (T*)(smem + S::OFF_WQ);
     T* la_all = (T*)(smem + S::OFF_LA);
     T* bt_s = (T*)(smem + S::OFF_BT);
@@ -481,6 +483,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         *sm_end = -1;
         *agg_done = 0;
         *(volatile int*)(smem + S::OFF_TAG + 12) = 0;
+        *lb_started = -1;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
@@ -548,7 +551,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
                 // (2) reload (from L2) the next tile whose carry is known, into a free carry buffer
                 if (j2 < j1 && j2 - j3 < NB2 &&
-                    mbar_test(SAM_EARLY_RELOAD ? &bar_p1[j2 % NQ] : &bar_carry[j2 % NQ], (uint32_t)((j2 / NQ) & 1))) {
+                    (SAM_EARLY_RELOAD == 2 ? (j2 / p.M <= *lb_started)
+                                           : mbar_test(SAM_EARLY_RELOAD ? &bar_p1[j2 % NQ] : &bar_carry[j2 % NQ],
+                                                       (uint32_t)((j2 / NQ) & 1)))) {
                     // groups committed after the store that last used this buffer (iteration j2-NB2)
                     const int later = j3 - 1 - (j2 - NB2);
                     if (later <= 0) bulk_wait_read<0>();
@@ -750,7 +755,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 __syncwarp();
                 if (lane == 0) cw_taken[bw] = r;
             }
-            if (lane == 0 && lead) SAM_TRACE(4, tile * p.M);
+            if (lane == 0 && lead) {
+                SAM_TRACE(4, tile * p.M);
+                if (SAM_EARLY_RELOAD == 2) *lb_started = r;  // its tiles may be re-fetched from L2 now
+            }
 
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, T* out) {
