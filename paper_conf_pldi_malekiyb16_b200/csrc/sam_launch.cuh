@@ -137,7 +137,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         uint64_t m = p.num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
         if (m < 1) m = 1;
         // measured: tuple 1: 3 (4-byte) / 2 (8-byte) tiles; tuples (more carry-team work per unit):
-        // 3, or 4 for odd tuples of 4-byte elements (i32 s=3: 4.5 -> 5.4 TB/s, s=5: 3.8 -> 5.5 TB/s)
+        // 3, or 4 for odd tuples of 4-byte elements (~1.5% better there)
         const uint64_t mmax = a.s == 1 ? (uint64_t)Lag<T, K>::MMAX : ((sizeof(T) == 4 && (a.s & 1)) ? 4u : 3u);
         if (m > mmax) m = mmax;
         if (const char* env = getenv("SAM_SUPER_TILE")) {  // experiments: force a smaller super-tile

@@ -10,8 +10,8 @@ cfgs = [("i32", 30, 1, 1), ("i32", 28, 1, 1), ("i64", 28, 1, 1), ("i32", 28, 2, 
         ("i64", 28, 1, 3), ("i64", 28, 1, 5), ("i64", 28, 1, 8), ("i64", 28, 2, 8), ("i64", 28, 4, 4),
         ("f32", 28, 1, 4), ("f64", 28, 1, 1)]
 if len(sys.argv) > 2:  # optional filter: "i32:30:1:1,i64:28:1:8"
-    want = {tuple(int(v) if i else v for i, v in enumerate(c.split(":"))) for c in sys.argv[2].split(",")}
-    cfgs = [c for c in cfgs if c in want] + [c for c in want if c not in cfgs]
+    want = [tuple(int(v) if i else v for i, v in enumerate(c.split(":"))) for c in sys.argv[2].split(",")]
+    cfgs = want  # in the order given
 data = {}
 for c in cfgs:
     dt, logn, k, s = c
