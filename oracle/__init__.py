@@ -5,6 +5,8 @@ import this package.  The product package (paper_conf_pldi_malekiyb16_b200) neve
 and it never imports the product package.
 
 scan(x, k, s, inclusive, phase=0, run=None) -> (y, run)
+delta(x, k, s) -> d       k-th order stride-s difference sequence (the encoder, P:1172-1186);
+                          same result dtypes as scan
     x      : 1-D numpy array, dtype int32 / int64 / float32 / float64
     y      : uint32 / uint64 (reinterpret as int32/int64 for comparisons), float64 for fp32
              data, np.longdouble for fp64 data
@@ -44,6 +46,10 @@ def _load():
         for name in ("oracle_scan_u32", "oracle_scan_u64", "oracle_scan_f64acc", "oracle_scan_ldacc"):
             fn = getattr(lib, name)
             fn.argtypes = [P, ctypes.c_uint64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P]
+            fn.restype = ctypes.c_int
+        for name in ("oracle_delta_u32", "oracle_delta_u64", "oracle_delta_f64acc", "oracle_delta_ldacc"):
+            fn = getattr(lib, name)
+            fn.argtypes = [P, ctypes.c_uint64, ctypes.c_int, ctypes.c_int]
             fn.restype = ctypes.c_int
         lib.oracle_sizeof_long_double.restype = ctypes.c_int
         _lib = lib
@@ -90,6 +96,23 @@ def scan_values(x: np.ndarray, k: int, s: int = 1, inclusive: bool = True) -> np
     if x.dtype.kind in "iu":
         return y.view(x.dtype)
     return y
+
+
+def delta(x: np.ndarray, k: int, s: int = 1) -> np.ndarray:
+    """k-th order stride-s difference sequence of x (k passes of first-order differencing,
+    missing values zero; sam_oracle.c oracle_delta_*).  Ints: uint32/uint64 result."""
+    lib = _load()
+    x = np.ascontiguousarray(x)
+    acc, fname = _ACC[x.dtype]
+    fname = fname.replace("oracle_scan_", "oracle_delta_")
+    if x.dtype.kind in "iu":
+        a = x.view(acc).copy() if x.dtype.itemsize == np.dtype(acc).itemsize else x.astype(acc)
+    else:
+        a = x.astype(acc)
+    rc = getattr(lib, fname)(a.ctypes.data, a.size, int(k), int(s))
+    if rc != 0:
+        raise ValueError(f"oracle rejected arguments (rc={rc}): k={k} s={s}")
+    return a
 
 
 def long_double_bytes() -> int:
