@@ -128,6 +128,21 @@ int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const v
 int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* all_payloads_host,
                            int rank, int nranks, void* seed_host);
 
+/*
+ * sam_delta_encode -- the k-th order, tuple-s difference sequence (delta ENCODER), the inverse of
+ * the inclusive sam_scan with the same (order, tuple):
+ *     out[i] = sum_{t=0..k} (-1)^t C(k,t) in[i - t*s],   in[j] = 0 for j < 0   ("missing" = 0)
+ * = first-order differencing out_i = in_i - in_{i-s} applied k times (Sec. 2.4; the
+ * paper's worked examples P:298-302; tuples P:349-355).  Embarrassingly parallel,
+ * one read and one write of HBM, one kernel launch.
+ *   dtype/order/tuple as for sam_scan; in, out: device pointers of n elements each.
+ *   Integers: exact mod 2^w.  fp32: accumulated in double, rounded once; fp64: double.
+ *   in == out (in place) or any overlap -> SAM_ERR_INVALID_ARG ("embarrassingly parallel when
+ *   not done in place").  n = 0 is a no-op.  Asynchronous on `stream`.
+ */
+int sam_delta_encode(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
+                     sam_stream_t stream);
+
 /* Diagnostics */
 const char* sam_last_error(void);
 const char* sam_version(void);

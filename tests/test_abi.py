@@ -74,6 +74,12 @@ def test_validation_invalid_args():
     assert L.sam_scan(0, 1, 1, 1, base, base + 8, 16, None) == -1               # partial overlap
     assert L.sam_shard_scan(0, 1, 1, 1, base, base + 256, 4, 0, base, 3, 2, None) == -1  # rank >= nranks
     assert L.sam_scan(0, 1, 1, 1, None, None, 0, None) == 0                     # n == 0 is a no-op
+    # delta encoder (not in place)
+    assert L.sam_delta_encode(0, 1, 1, base, base, 4, None) == -1               # in place refused
+    assert L.sam_delta_encode(0, 1, 1, base, base + 8, 16, None) == -1          # partial overlap
+    assert L.sam_delta_encode(0, 9, 1, base, base + 256, 4, None) == -2         # order > 8
+    assert L.sam_delta_encode(0, 1, 0, base, base + 256, 4, None) == -2         # tuple < 1
+    assert L.sam_delta_encode(3, 1, 1, None, None, 0, None) == 0                # n == 0 is a no-op
 
 
 @pytest.mark.parametrize("dt,k,s,expected", [(0, 1, 1, 32), (1, 4, 4, 144), (1, 8, 8, 528), (2, 3, 5, 80)])
