@@ -12,7 +12,9 @@
 // coalesced loads (evict-first: every element is read from HBM once) behind a halo of the k*s <= 64
 // preceding elements (plain loads: the previous tile's bytes, likely still in L2).  Each thread
 // then evaluates the stencil for elements j = e*THREADS + tid (conflict-free 32-bit LDS, stride 1
-// across a warp) and writes them with coalesced streaming stores.  Integers: unsigned arithmetic
+// across a warp) and writes them with coalesced streaming stores; for s = 1 it instead slides a
+// register window of 128-bit vectors (k + 1 smem reads per element would make orders >= 8 bound by
+// shared-memory bandwidth rather than HBM).  Integers: unsigned arithmetic
 // mod 2^w (the identity holds in the ring Z/2^w, so the result equals k passes of first-order
 // differencing bit for bit); fp32: accumulated in double, rounded once; fp64: accumulated in double.
 #include <cuda_runtime.h>
@@ -38,7 +40,7 @@ template <typename T> __device__ __forceinline__ T zero_of() { return T(0); }
 
 template <typename T, int K>
 __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ in, T* __restrict__ out,
-                                                           uint64_t n, int s, int vec_ok) {
+                                                           uint64_t n, int s, int vec_ok /* bit0 in, bit1 out 16-B aligned */) {
     using G = DeltaGeom<T>;
     using A = typename DeltaAcc<T>::type;
     __shared__ __align__(16) T sm[D_HALO + G::TILE];
@@ -63,7 +65,7 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         const uint64_t q = (uint64_t)tid + 1;
         sm[D_HALO - (int)q] = (b >= q) ? in[b - q] : zero_of<T>();
     }
-    if (vec_ok && cnt == G::TILE) {
+    if ((vec_ok & 1) && cnt == G::TILE) {
         const int4* src = reinterpret_cast<const int4*>(in + b);
         int4* dst = reinterpret_cast<int4*>(sm + D_HALO);
         int4 v[G::VPT];
@@ -75,6 +77,39 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         for (int j = tid; j < cnt; j += D_THREADS) sm[D_HALO + j] = __ldcs(in + b + j);
     }
     __syncthreads();
+
+    if (s == 1 && (vec_ok & 2) && cnt == G::TILE) {
+        // s = 1, full tile: thread tid owns the 128-bit vectors u*THREADS + tid and reads each one
+        // with the NH vectors before it (LDS.128, consecutive threads on consecutive vectors:
+        // conflict free) into a register window; the stencil then runs on registers, so shared
+        // memory carries (NH + 1) * 16 B per V outputs instead of (K + 1) * w per output.
+        constexpr int V = G::V;
+        constexpr int NH = (K + V - 1) / V;  // <= D_HALO / V, so the window stays inside sm
+        const int4* sv = reinterpret_cast<const int4*>(sm + D_HALO);
+        int4* ov = reinterpret_cast<int4*>(out + b);
+#pragma unroll
+        for (int u = 0; u < G::VPT; ++u) {
+            const int vi = u * D_THREADS + tid;
+            T win[(NH + 1) * V];
+#pragma unroll
+            for (int h = 0; h <= NH; ++h) {
+                const int4 q = sv[vi - NH + h];
+                const T* qt = reinterpret_cast<const T*>(&q);
+#pragma unroll
+                for (int e = 0; e < V; ++e) win[h * V + e] = qt[e];
+            }
+            T r[V];
+#pragma unroll
+            for (int e = 0; e < V; ++e) {
+                A acc = (A)win[NH * V + e];
+#pragma unroll
+                for (int t = 1; t <= K; ++t) acc = acc + c[t] * (A)win[NH * V + e - t];
+                r[e] = (T)acc;
+            }
+            __stcs(ov + vi, *reinterpret_cast<const int4*>(r));
+        }
+        return;
+    }
 
 #pragma unroll 4
     for (int e = 0; e < G::PER_THREAD; ++e) {
@@ -93,7 +128,7 @@ template <typename T, int K>
 cudaError_t launch_k(const T* in, T* out, uint64_t n, int s, cudaStream_t st) {
     using G = DeltaGeom<T>;
     const uint64_t tiles = (n + G::TILE - 1) / G::TILE;
-    const int vec_ok = ((uintptr_t)in % 16) == 0;
+    const int vec_ok = (((uintptr_t)in % 16) == 0 ? 1 : 0) | (((uintptr_t)out % 16) == 0 ? 2 : 0);
     delta_kernel<T, K><<<(unsigned)tiles, D_THREADS, 0, st>>>(in, out, n, s, vec_ok);
     return cudaGetLastError();
 }
