@@ -143,6 +143,14 @@ int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* al
 int sam_delta_encode(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
                      sam_stream_t stream);
 
+/* sam_delta_encode of a chunk / shard that continues an earlier stream: `halo` is a device
+ * pointer to the order*tuple elements immediately preceding in[0] (halo[order*tuple - 1] is
+ * adjacent to in[0]; zero-padded on the left when fewer precede), NULL = none ("missing" values
+ * zero).  Encoding the shards of an array with their halos gives exactly the
+ * whole-array result.  Misaligned halo -> SAM_ERR_INVALID_ARG. */
+int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
+                          const void* halo, sam_stream_t stream);
+
 /* Diagnostics */
 const char* sam_last_error(void);
 const char* sam_version(void);

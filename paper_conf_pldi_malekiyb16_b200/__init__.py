@@ -17,7 +17,7 @@ __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
     "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
-    "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
+    "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
 ]
 
 SAM_I32, SAM_I64, SAM_F32, SAM_F64 = 0, 1, 2, 3
@@ -54,6 +54,7 @@ def lib() -> ctypes.CDLL:
             "sam_shard_scan": (I, [I, I, I, I, P, P, U64, U64, P, I, I, P]),
             "sam_fold_payloads_host": (I, [I, I, I, P, I, I, P]),
             "sam_delta_encode": (I, [I, I, I, P, P, U64, P]),
+            "sam_delta_encode_halo": (I, [I, I, I, P, P, U64, P, P]),
             "sam_last_error": (ctypes.c_char_p, []),
             "sam_version": (ctypes.c_char_p, []),
             "sam_release_workspaces": (I, []),
@@ -116,6 +117,10 @@ def sam_delta_encode(dtype, order, tuple_, in_ptr, out_ptr, n, stream=None) -> i
     return _check(lib().sam_delta_encode(dtype, order, tuple_, in_ptr, out_ptr, n, stream))
 
 
+def sam_delta_encode_halo(dtype, order, tuple_, in_ptr, out_ptr, n, halo_ptr, stream=None) -> int:
+    return _check(lib().sam_delta_encode_halo(dtype, order, tuple_, in_ptr, out_ptr, n, halo_ptr, stream))
+
+
 def sam_last_error() -> str:
     return lib().sam_last_error().decode()
 
@@ -165,17 +170,24 @@ def scan(x, order: int = 1, tuple: int = 1, inclusive: bool = True, out=None, st
     return out
 
 
-def delta_encode(x, order: int = 1, tuple: int = 1, out=None, stream=None):
+def delta_encode(x, order: int = 1, tuple: int = 1, out=None, stream=None, halo=None):
     """Order-`order`, tuple-`tuple` difference sequence of a 1-D contiguous CUDA tensor
-    (sam_delta_encode): the inverse of scan(..., inclusive=True).  Not in place."""
+    (sam_delta_encode): the inverse of scan(..., inclusive=True).  Not in place.
+    `halo`: optional CUDA tensor of the order*tuple elements preceding x (sam_delta_encode_halo)."""
     if not x.is_cuda or x.dim() != 1 or not x.is_contiguous():
         raise SamError(-1, "delta_encode() needs a 1-D contiguous CUDA tensor")
     if out is None:
         import torch
 
         out = torch.empty_like(x)
-    sam_delta_encode(dtype_code(x.dtype), order, tuple, ctypes.c_void_p(x.data_ptr()),
-                     ctypes.c_void_p(out.data_ptr()), x.numel(), _stream_ptr(stream))
+    if halo is not None:
+        if not halo.is_cuda or halo.dtype != x.dtype or halo.numel() != order * tuple or not halo.is_contiguous():
+            raise SamError(-1, "halo must be a contiguous CUDA tensor of order*tuple elements of x's dtype")
+        hp = ctypes.c_void_p(halo.data_ptr())
+    else:
+        hp = None
+    sam_delta_encode_halo(dtype_code(x.dtype), order, tuple, ctypes.c_void_p(x.data_ptr()),
+                          ctypes.c_void_p(out.data_ptr()), x.numel(), hp, _stream_ptr(stream))
     return out
 
 

@@ -18,7 +18,7 @@
 
 namespace sam {
 template <typename T, int K> cudaError_t launch_scan_tk(const LaunchArgs&, uint64_t*);
-template <typename T> cudaError_t launch_delta(const void*, void*, uint64_t, int, int, cudaStream_t, uint64_t*);
+template <typename T> cudaError_t launch_delta(const void*, void*, uint64_t, int, int, const void*, cudaStream_t, uint64_t*);
 template <typename T> cudaError_t launch_fold(const void*, size_t, int, int, int, void*, cudaStream_t, uint64_t*);
 template <typename T> cudaError_t launch_payload_init(void*, uint64_t, uint64_t, int, int, const void*, int, void*,
                                                       cudaStream_t, uint64_t*);
@@ -423,6 +423,11 @@ int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const vo
 
 int sam_delta_encode(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
                      sam_stream_t stream) {
+    return sam_delta_encode_halo(dtype, order, tuple, in, out, n, nullptr, stream);
+}
+
+int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
+                          const void* halo, sam_stream_t stream) {
     int rc = validate_common(dtype, order, tuple);
     if (rc) return rc;
     rc = validate_buffers(dtype, in, out, n, true);
@@ -430,14 +435,16 @@ int sam_delta_encode(sam_dtype dtype, int order, int tuple, const void* in, void
     if (n > 0 && in == out)
         return fail(SAM_ERR_INVALID_ARG, "delta encoding is not done in place (P:281-284): in must differ from out");
     if (n == 0) return SAM_OK;
+    if (halo && ((uintptr_t)halo % elem_size(dtype)) != 0)
+        return fail(SAM_ERR_INVALID_ARG, "halo must be aligned to the element size");
     cudaStream_t st = (cudaStream_t)stream;
     uint64_t l = 0;
     cudaError_t e;
     switch (dtype) {
-        case SAM_I32: e = sam::launch_delta<uint32_t>(in, out, n, order, tuple, st, &l); break;
-        case SAM_I64: e = sam::launch_delta<uint64_t>(in, out, n, order, tuple, st, &l); break;
-        case SAM_F32: e = sam::launch_delta<float>(in, out, n, order, tuple, st, &l); break;
-        default: e = sam::launch_delta<double>(in, out, n, order, tuple, st, &l); break;
+        case SAM_I32: e = sam::launch_delta<uint32_t>(in, out, n, order, tuple, halo, st, &l); break;
+        case SAM_I64: e = sam::launch_delta<uint64_t>(in, out, n, order, tuple, halo, st, &l); break;
+        case SAM_F32: e = sam::launch_delta<float>(in, out, n, order, tuple, halo, st, &l); break;
+        default: e = sam::launch_delta<double>(in, out, n, order, tuple, halo, st, &l); break;
     }
     g_launches += l;
     return e == cudaSuccess ? SAM_OK : cuda_fail(e, "delta encoder launch");

@@ -40,7 +40,8 @@ template <typename T> __device__ __forceinline__ T zero_of() { return T(0); }
 
 template <typename T, int K>
 __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ in, T* __restrict__ out,
-                                                           uint64_t n, int s, int vec_ok /* bit0 in, bit1 out 16-B aligned */) {
+                                                           uint64_t n, int s, int vec_ok /* bit0 in, bit1 out 16-B aligned */,
+                                                           const T* __restrict__ halo) {
     using G = DeltaGeom<T>;
     using A = typename DeltaAcc<T>::type;
     __shared__ __align__(16) T sm[D_HALO + G::TILE];
@@ -63,7 +64,8 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
 
     if (tid < ks) {
         const uint64_t q = (uint64_t)tid + 1;
-        sm[D_HALO - (int)q] = (b >= q) ? in[b - q] : zero_of<T>();
+        // before in[0]: the caller's halo (halo[ks-1] adjacent to in[0]) or "missing" = 0
+        sm[D_HALO - (int)q] = (b >= q) ? in[b - q] : (halo ? halo[ks - (int)(q - b)] : zero_of<T>());
     }
     if ((vec_ok & 1) && cnt == G::TILE) {
         const int4* src = reinterpret_cast<const int4*>(in + b);
@@ -125,43 +127,44 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
 }
 
 template <typename T, int K>
-cudaError_t launch_k(const T* in, T* out, uint64_t n, int s, cudaStream_t st) {
+cudaError_t launch_k(const T* in, T* out, uint64_t n, int s, const T* halo, cudaStream_t st) {
     using G = DeltaGeom<T>;
     const uint64_t tiles = (n + G::TILE - 1) / G::TILE;
     const int vec_ok = (((uintptr_t)in % 16) == 0 ? 1 : 0) | (((uintptr_t)out % 16) == 0 ? 2 : 0);
-    delta_kernel<T, K><<<(unsigned)tiles, D_THREADS, 0, st>>>(in, out, n, s, vec_ok);
+    delta_kernel<T, K><<<(unsigned)tiles, D_THREADS, 0, st>>>(in, out, n, s, vec_ok, halo);
     return cudaGetLastError();
 }
 
 }  // namespace
 
-// One launch of the delta encoder (n > 0, 1 <= k, s <= 8, in/out non-overlapping, validated by
+// One launch of the delta encoder (halo: NULL or k*s elements preceding in[0]; n > 0, 1 <= k, s <= 8, in/out non-overlapping, validated by
 // the caller).  *launches is incremented by the number of kernels launched.
 template <typename T>
-cudaError_t launch_delta(const void* in_, void* out_, uint64_t n, int k, int s, cudaStream_t st,
-                         uint64_t* launches) {
+cudaError_t launch_delta(const void* in_, void* out_, uint64_t n, int k, int s, const void* halo_,
+                         cudaStream_t st, uint64_t* launches) {
+    const T* halo = (const T*)halo_;
     const T* in = (const T*)in_;
     T* out = (T*)out_;
     if (n == 0) return cudaSuccess;
     if ((n + DeltaGeom<T>::TILE - 1) / DeltaGeom<T>::TILE > 0x7fffffffull) return cudaErrorInvalidValue;
     cudaError_t e = cudaErrorInvalidValue;
     switch (k) {
-        case 1: e = launch_k<T, 1>(in, out, n, s, st); break;
-        case 2: e = launch_k<T, 2>(in, out, n, s, st); break;
-        case 3: e = launch_k<T, 3>(in, out, n, s, st); break;
-        case 4: e = launch_k<T, 4>(in, out, n, s, st); break;
-        case 5: e = launch_k<T, 5>(in, out, n, s, st); break;
-        case 6: e = launch_k<T, 6>(in, out, n, s, st); break;
-        case 7: e = launch_k<T, 7>(in, out, n, s, st); break;
-        case 8: e = launch_k<T, 8>(in, out, n, s, st); break;
+        case 1: e = launch_k<T, 1>(in, out, n, s, halo, st); break;
+        case 2: e = launch_k<T, 2>(in, out, n, s, halo, st); break;
+        case 3: e = launch_k<T, 3>(in, out, n, s, halo, st); break;
+        case 4: e = launch_k<T, 4>(in, out, n, s, halo, st); break;
+        case 5: e = launch_k<T, 5>(in, out, n, s, halo, st); break;
+        case 6: e = launch_k<T, 6>(in, out, n, s, halo, st); break;
+        case 7: e = launch_k<T, 7>(in, out, n, s, halo, st); break;
+        case 8: e = launch_k<T, 8>(in, out, n, s, halo, st); break;
     }
     if (e == cudaSuccess) *launches += 1;
     return e;
 }
 
-template cudaError_t launch_delta<uint32_t>(const void*, void*, uint64_t, int, int, cudaStream_t, uint64_t*);
-template cudaError_t launch_delta<uint64_t>(const void*, void*, uint64_t, int, int, cudaStream_t, uint64_t*);
-template cudaError_t launch_delta<float>(const void*, void*, uint64_t, int, int, cudaStream_t, uint64_t*);
-template cudaError_t launch_delta<double>(const void*, void*, uint64_t, int, int, cudaStream_t, uint64_t*);
+template cudaError_t launch_delta<uint32_t>(const void*, void*, uint64_t, int, int, const void*, cudaStream_t, uint64_t*);
+template cudaError_t launch_delta<uint64_t>(const void*, void*, uint64_t, int, int, const void*, cudaStream_t, uint64_t*);
+template cudaError_t launch_delta<float>(const void*, void*, uint64_t, int, int, const void*, cudaStream_t, uint64_t*);
+template cudaError_t launch_delta<double>(const void*, void*, uint64_t, int, int, const void*, cudaStream_t, uint64_t*);
 
 }  // namespace sam

@@ -11,6 +11,12 @@ One process per GPU.  Rank r holds elements [g_r, g_r + n_r) of the global array
                          (M(L) s + v) into this shard's seed, then the seeded
                          single-pass scan (binomial fix-up fused into the carry application)
 
+Sharded delta ENCODER: each rank needs the order*tuple elements before its
+shard.  Every rank contributes the last min(n_r, 64) elements of its shard (TAIL = 64 >= max k*s)
+and n_r to one all-gather; rank r's halo is the last k*s elements of the concatenated valid tails
+of ranks < r (left-padded with zeros), then sam_delta_encode_halo encodes the shard.  Pure data
+movement on the host side; the differencing runs in the library's kernel.
+
 torch.distributed is plumbing only; every arithmetic step runs in libsam.so kernels.
 """
 from __future__ import annotations
@@ -20,7 +26,10 @@ import ctypes
 import torch
 import torch.distributed as dist
 
-from . import (SamError, _stream_ptr, dtype_code, sam_shard_payload_bytes, sam_shard_scan, sam_shard_state)
+from . import (SamError, _stream_ptr, delta_encode, dtype_code, sam_shard_payload_bytes, sam_shard_scan,
+               sam_shard_state)
+
+TAIL = 64  # elements each rank contributes to the halo exchange (>= max order*tuple = 64)
 
 
 def shard_offsets(n_local: int, group=None, device=None) -> tuple[int, int]:
@@ -93,4 +102,59 @@ def scan_virtual_shards(x: torch.Tensor, bounds: list[int], order: int = 1, tupl
         sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x.data_ptr() + lo * w),
                        ctypes.c_void_p(out.data_ptr() + lo * w), hi - lo, lo,
                        ctypes.c_void_p(gathered.data_ptr()), r, p, st)
+    return out
+
+
+# ----------------------------------------------------------------------------- delta encoder
+def shard_tail(x_local: torch.Tensor) -> torch.Tensor:
+    """The last min(n, TAIL) elements of a shard, right-aligned in a zero tensor of TAIL."""
+    t = torch.zeros(TAIL, dtype=x_local.dtype, device=x_local.device)
+    m = min(x_local.numel(), TAIL)
+    if m:
+        t[TAIL - m:] = x_local[x_local.numel() - m:]
+    return t
+
+
+def halo_from_tails(tails: torch.Tensor, lens: list[int], rank: int, ks: int) -> torch.Tensor:
+    """Halo of `rank` (the ks elements preceding its shard, zero-left-padded) from the gathered
+    tails [world, TAIL] and shard lengths: the suffix of the valid tails of ranks < rank.  The
+    valid tail of a shard is all of it when n < TAIL, so the concatenation ends with the last
+    TAIL elements of the global prefix."""
+    parts = [tails[r, TAIL - min(lens[r], TAIL):] for r in range(rank)]
+    z = torch.zeros(ks, dtype=tails.dtype, device=tails.device)
+    cat = torch.cat([z] + parts)
+    return cat[cat.numel() - ks:].contiguous()
+
+
+def delta_encode_sharded(x_local: torch.Tensor, order: int = 1, tuple: int = 1, group=None,
+                         out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Delta encoding (k-th order, stride s) of the global array whose contiguous shard `x_local`
+    this rank holds: one all-gather of shard tails and lengths, then sam_delta_encode_halo."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    if world == 1:
+        return delta_encode(x_local, order, tuple, out=out, stream=stream)
+    tail = shard_tail(x_local)
+    tails = torch.empty(world * TAIL, dtype=x_local.dtype, device=x_local.device)
+    dist.all_gather_into_tensor(tails, tail, group=group)
+    tails = tails.view(world, TAIL)
+    n = torch.tensor([x_local.numel()], dtype=torch.int64, device=x_local.device)
+    lens_t = torch.empty(world, dtype=torch.int64, device=x_local.device)
+    dist.all_gather_into_tensor(lens_t, n, group=group)
+    halo = halo_from_tails(tails, lens_t.tolist(), rank, order * tuple)
+    return delta_encode(x_local, order, tuple, out=out, stream=stream, halo=halo)
+
+
+def delta_virtual_shards(x: torch.Tensor, bounds: list[int], order: int = 1, tuple: int = 1) -> torch.Tensor:
+    """The sharded encoder's schedule on ONE GPU over virtual shards x[bounds[i]:bounds[i+1]]
+    (tail stacking in place of the all-gather)."""
+    p = len(bounds) - 1
+    shards = [x[bounds[r]:bounds[r + 1]] for r in range(p)]
+    tails = torch.stack([shard_tail(sh) for sh in shards])
+    lens = [sh.numel() for sh in shards]
+    out = torch.empty_like(x)
+    for r in range(p):
+        if lens[r]:
+            delta_encode(shards[r], order, tuple, out=out[bounds[r]:bounds[r + 1]],
+                         halo=halo_from_tails(tails, lens, r, order * tuple))
     return out
