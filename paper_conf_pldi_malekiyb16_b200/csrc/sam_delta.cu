@@ -13,8 +13,9 @@
 // preceding elements (plain loads: the previous tile's bytes, likely still in L2).  Each thread
 // then evaluates the stencil for elements j = e*THREADS + tid (conflict-free 32-bit LDS, stride 1
 // across a warp) and writes them with coalesced streaming stores; for s = 1 it instead slides a
-// register window of 128-bit vectors (k + 1 smem reads per element would make orders >= 8 bound by
-// shared-memory bandwidth rather than HBM).  Integers: unsigned arithmetic
+// register window of 128-bit vectors, and for s > 1 with k*s >= 24 each thread walks one lane of
+// a chunk with the lane's last k values in a shift register (k + 1 smem reads per element would
+// make high orders bound by shared-memory bandwidth rather than HBM).  Integers: unsigned arithmetic
 // mod 2^w (the identity holds in the ring Z/2^w, so the result equals k passes of first-order
 // differencing bit for bit); fp32: accumulated in double, rounded once; fp64: accumulated in double.
 #include <cuda_runtime.h>
@@ -25,6 +26,7 @@ namespace {
 
 constexpr int D_THREADS = 256;
 constexpr int D_HALO = 64;  // >= max k*s = 8*8
+constexpr int D_LANE_MIN_KS = 24;  // k*s from which s > 1 takes the lane-strided register path
 
 template <typename T> struct DeltaAcc { using type = T; };
 template <> struct DeltaAcc<float> { using type = double; };
@@ -109,6 +111,39 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
                 r[e] = (T)acc;
             }
             __stcs(ov + vi, *reinterpret_cast<const int4*>(r));
+        }
+        return;
+    }
+
+    if (s > 1 && ks >= D_LANE_MIN_KS) {
+        // large k*s: lane-strided register path.  Unit u = (chunk c, lane m) owns the R positions
+        // c*s*R + m + i*s (i < R) of one lane and keeps the K previous values of that lane in a
+        // shift register, so a unit reads R + K smem values for R outputs instead of (K + 1) * R.
+        // R odd (17 / 9) keeps the warp's reads on distinct banks for even s, and
+        // ceil(TILE / (s R)) * s <= 256 units, so one pass of the block covers the tile.
+        constexpr int R = sizeof(T) == 4 ? 17 : 9;
+        const int span = s * R;
+        const int nunits = ((cnt + span - 1) / span) * s;
+        for (int u = tid; u < nunits; u += D_THREADS) {
+            const int cc = u / s;
+            const int p0 = cc * span + (u - cc * s);
+            A h[K];  // h[t-1] = x[p - t*s]
+#pragma unroll
+            for (int t = 1; t <= K; ++t) h[t - 1] = (A)sm[D_HALO + p0 - t * s];
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const int p = p0 + i * s;
+                if (p < cnt) {
+                    const A xv = (A)sm[D_HALO + p];
+                    A acc = xv;
+#pragma unroll
+                    for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
+                    __stcs(out + b + p, (T)acc);
+#pragma unroll
+                    for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
+                    h[0] = xv;
+                }
+            }
         }
         return;
     }
