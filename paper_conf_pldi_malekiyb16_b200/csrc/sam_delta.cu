@@ -120,30 +120,50 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         // c*s*R + m + i*s (i < R) of one lane and keeps the K previous values of that lane in a
         // shift register, so a unit reads R + K smem values for R outputs instead of (K + 1) * R.
         // R odd (17 / 9) keeps the warp's reads on distinct banks for even s, and
-        // ceil(TILE / (s R)) * s <= 256 units, so one pass of the block covers the tile.
+        // ceil(TILE / (s R)) * s <= 248 (4-byte) / 232 (8-byte) units for every s <= 8: one unit
+        // per thread covers the tile.
         constexpr int R = sizeof(T) == 4 ? 17 : 9;
         const int span = s * R;
-        const int nunits = ((cnt + span - 1) / span) * s;
-        for (int u = tid; u < nunits; u += D_THREADS) {
-            const int cc = u / s;
-            const int p0 = cc * span + (u - cc * s);
+        const int nunits = ((cnt + span - 1) / span) * s;  // <= D_THREADS (see above)
+        const int u = tid;
+        const int cc = u / s;
+        const int p0 = cc * span + (u - cc * s);
+        T r[R];
+        if (u < nunits) {
             A h[K];  // h[t-1] = x[p - t*s]
 #pragma unroll
             for (int t = 1; t <= K; ++t) h[t - 1] = (A)sm[D_HALO + p0 - t * s];
 #pragma unroll
             for (int i = 0; i < R; ++i) {
                 const int p = p0 + i * s;
-                if (p < cnt) {
-                    const A xv = (A)sm[D_HALO + p];
-                    A acc = xv;
+                const A xv = (p < cnt) ? (A)sm[D_HALO + p] : (A)0;
+                A acc = xv;
 #pragma unroll
-                    for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
-                    __stcs(out + b + p, (T)acc);
+                for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
+                r[i] = (T)acc;
 #pragma unroll
-                    for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
-                    h[0] = xv;
-                }
+                for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
+                h[0] = xv;
             }
+        }
+        // the outputs go back through shared memory so the global stores stay coalesced (a warp's
+        // direct stores would be s-element groups at stride s*R: partial sectors for most s)
+        __syncthreads();
+        if (u < nunits) {
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const int p = p0 + i * s;
+                if (p < cnt) sm[D_HALO + p] = r[i];
+            }
+        }
+        __syncthreads();
+        if ((vec_ok & 2) && cnt == G::TILE) {
+            const int4* src = reinterpret_cast<const int4*>(sm + D_HALO);
+            int4* dst = reinterpret_cast<int4*>(out + b);
+#pragma unroll
+            for (int v = 0; v < G::VPT; ++v) __stcs(dst + v * D_THREADS + tid, src[v * D_THREADS + tid]);
+        } else {
+            for (int j = tid; j < cnt; j += D_THREADS) __stcs(out + b + j, sm[D_HALO + j]);
         }
         return;
     }
