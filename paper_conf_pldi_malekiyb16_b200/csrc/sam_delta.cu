@@ -128,32 +128,30 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         const int u = tid;
         const int cc = u / s;
         const int p0 = cc * span + (u - cc * s);
-        T r[R];
+        // A unit's only reads of other units' values are its K history values (the previous chunk
+        // of its lane): take them, then after one barrier each unit owns its R positions alone and
+        // overwrites them in place with its outputs, which then leave through coalesced 128-bit
+        // stores (a warp's direct stores would be s-element groups at stride s*R: partial sectors).
+        A h[K];  // h[t-1] = x[p - t*s]
         if (u < nunits) {
-            A h[K];  // h[t-1] = x[p - t*s]
 #pragma unroll
             for (int t = 1; t <= K; ++t) h[t - 1] = (A)sm[D_HALO + p0 - t * s];
-#pragma unroll
-            for (int i = 0; i < R; ++i) {
-                const int p = p0 + i * s;
-                const A xv = (p < cnt) ? (A)sm[D_HALO + p] : (A)0;
-                A acc = xv;
-#pragma unroll
-                for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
-                r[i] = (T)acc;
-#pragma unroll
-                for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
-                h[0] = xv;
-            }
         }
-        // the outputs go back through shared memory so the global stores stay coalesced (a warp's
-        // direct stores would be s-element groups at stride s*R: partial sectors for most s)
         __syncthreads();
         if (u < nunits) {
 #pragma unroll
             for (int i = 0; i < R; ++i) {
                 const int p = p0 + i * s;
-                if (p < cnt) sm[D_HALO + p] = r[i];
+                if (p < cnt) {
+                    const A xv = (A)sm[D_HALO + p];
+                    A acc = xv;
+#pragma unroll
+                    for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
+                    sm[D_HALO + p] = (T)acc;
+#pragma unroll
+                    for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
+                    h[0] = xv;
+                }
             }
         }
         __syncthreads();
