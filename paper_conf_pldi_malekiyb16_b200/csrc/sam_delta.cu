@@ -139,52 +139,18 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         }
         __syncthreads();
         if (u < nunits) {
-            if constexpr (sizeof(A) == sizeof(T) && (T)(-1) > (T)0) {
-                // integers: the difference cascade (k subtractions per output instead of k
-                // multiply-adds; equal mod 2^w).  g[t] = Delta^t x at the lane's previous position,
-                // formed by running the cascade over the K history values, oldest first: Delta^t
-                // there needs only t <= K-1 older values, all in h.
-                T g[K];
 #pragma unroll
-                for (int t = 0; t < K; ++t) g[t] = 0;
+            for (int i = 0; i < R; ++i) {
+                const int p = p0 + i * s;
+                if (p < cnt) {
+                    const A xv = (A)sm[D_HALO + p];
+                    A acc = xv;
 #pragma unroll
-                for (int j = K - 1; j >= 0; --j) {
-                    T v = h[j];
+                    for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
+                    sm[D_HALO + p] = (T)acc;
 #pragma unroll
-                    for (int t = 0; t < K; ++t) {
-                        const T nv = v - g[t];
-                        g[t] = v;
-                        v = nv;
-                    }
-                }
-#pragma unroll
-                for (int i = 0; i < R; ++i) {
-                    const int p = p0 + i * s;
-                    if (p < cnt) {
-                        T v = sm[D_HALO + p];
-#pragma unroll
-                        for (int t = 0; t < K; ++t) {
-                            const T nv = v - g[t];
-                            g[t] = v;
-                            v = nv;
-                        }
-                        sm[D_HALO + p] = v;
-                    }
-                }
-            } else {
-#pragma unroll
-                for (int i = 0; i < R; ++i) {
-                    const int p = p0 + i * s;
-                    if (p < cnt) {
-                        const A xv = (A)sm[D_HALO + p];
-                        A acc = xv;
-#pragma unroll
-                        for (int t = 1; t <= K; ++t) acc = acc + c[t] * h[t - 1];
-                        sm[D_HALO + p] = (T)acc;
-#pragma unroll
-                        for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
-                        h[0] = xv;
-                    }
+                    for (int t = K - 1; t > 0; --t) h[t] = h[t - 1];
+                    h[0] = xv;
                 }
             }
         }
