@@ -38,7 +38,14 @@ CONFIGS = {
     "C3i64k8": ("i64", 28, 8, 1, True, "C3: n=2^28 int64 order-8 tuple-1 inclusive scan"),
     "C4s8": ("i64", 28, 1, 8, True, "C4: n=2^28 int64 order-1 tuple-8 inclusive scan"),
     "C5": ("i64", 30, 4, 4, True, "C5: int64 order-4 tuple-4 inclusive scan, 2^30 per GPU"),
+    # the encoder, not the north-star path: --config D2 / D2k8
+    "D2": ("i32", 30, 1, 1, True, "D2: n=2^30 int32 order-1 tuple-1 delta ENCODE (sam_delta_encode, NEXT-2)"),
+    "D2k8": ("i32", 30, 8, 1, True, "D2k8: n=2^30 int32 order-8 tuple-1 delta ENCODE (sam_delta_encode, NEXT-2)"),
 }
+
+
+def is_delta(config_name):
+    return config_name.startswith("D")
 W_BYTES = {"i32": 4, "i64": 8, "f32": 4, "f64": 8}
 DTYPE_NAME = {"i32": "int32", "i64": "int64", "f32": "float32", "f64": "float64"}
 
@@ -136,13 +143,14 @@ def run_reference(args):
     n_total = (1 << logn) * max(1, args.gpus)
     sample = min(n_total, 1 << 27)  # bounded: ~0.1-1 s of serial CPU work per step
     x = synth.make(sample, dt, "uniform", seed=synth.SEED_BASE + 1)
-    oracle.scan(x[: 1 << 16], k, s, incl)
+    run = (lambda a: oracle.delta(a, k, s)) if is_delta(args.config) else (lambda a: oracle.scan(a, k, s, incl))
+    run(x[: 1 << 16])
     for _ in range(args.warmup):
-        oracle.scan(x[: 1 << 20], k, s, incl)
+        run(x[: 1 << 20])
     times = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        oracle.scan(x, k, s, incl)
+        run(x)
         times.append(time.perf_counter() - t0)
     t = statistics.median(times)
     gv = sample / t / 1e9
@@ -205,8 +213,21 @@ def main():
     ev_k1 = torch.cuda.Event(enable_timing=True)
     kern_ms = []
 
+    delta = is_delta(args.config)
+    if delta and world > 1:
+        from paper_conf_pldi_malekiyb16_b200.dist import delta_encode_sharded
+
     def step(time_kernel=False):
-        if world == 1:
+        if delta:
+            if time_kernel:
+                ev_k0.record(stream)
+            if world == 1:
+                sam.sam_delta_encode(dc, k, s, P(x), P(y), n_local, sp)
+            else:
+                delta_encode_sharded(x, k, s, out=y)
+            if time_kernel:
+                ev_k1.record(stream)
+        elif world == 1:
             if time_kernel:
                 ev_k0.record(stream)
             sam.sam_scan(dc, k, s, incl, P(x), P(y), n_local, sp)
@@ -278,7 +299,7 @@ def main():
         import oracle
 
         m = 1 << 20
-        ref = oracle.scan(x[:m].cpu().numpy(), k, s, incl)[0]
+        ref = oracle.delta(x[:m].cpu().numpy(), k, s) if delta else oracle.scan(x[:m].cpu().numpy(), k, s, incl)[0]
         got = y[:m].cpu().numpy().view(ref.dtype)
         check = bool(np.array_equal(got, ref))
 
@@ -287,7 +308,29 @@ def main():
     if not args.no_e2e:
         xh = x.cpu().pin_memory()
         yh = torch.empty_like(xh).pin_memory()
-        if world == 1:
+        if delta:
+            # encoder e2e: pinned H2D, sam_delta_encode (halo-exchanged under torchrun), D2H
+            xd = torch.empty_like(x)
+            yd = torch.empty_like(x)
+            tt = []
+            for _ in range(4):
+                if world > 1:
+                    dist.barrier()
+                t0 = time.perf_counter()
+                xd.copy_(xh, non_blocking=True)
+                if world == 1:
+                    sam.sam_delta_encode(dc, k, s, P(xd), P(yd), n_local, sp)
+                else:
+                    delta_encode_sharded(xd, k, s, out=yd)
+                yh.copy_(yd, non_blocking=True)
+                torch.cuda.synchronize()
+                tt.append(time.perf_counter() - t0)
+            tte = torch.tensor([statistics.median(tt[1:])], dtype=torch.float64, device=dev)
+            if world > 1:
+                dist.all_reduce(tte, op=dist.ReduceOp.MAX)
+            te = float(tte[0])
+            del xd, yd
+        elif world == 1:
             sam.sam_scan_host(dc, k, s, incl, P(xh), P(yh), n_local, sp)
             reps = 3
             tt = []
@@ -315,7 +358,8 @@ def main():
             te = float(tte[0])
         e2e = {"value": n_total / te / 1e9, "unit": "Gvalues/s", "h2d_bytes_per_step": n_local * w * world,
                "d2h_bytes_per_step": n_local * w * world, "ms_per_step": te * 1e3,
-               "path": "sam_scan_host: pinned host buffers, 128 MiB chunks, H2D | seeded scan | D2H on 3 streams"
+               "path": "pinned H2D, sam_delta_encode, D2H (serial)" if delta else
+               "sam_scan_host: pinned host buffers, 128 MiB chunks, H2D | seeded scan | D2H on 3 streams"
                if world == 1 else "per rank: pinned H2D, shard state, NCCL all-gather, shard scan, D2H"}
 
     # CPU oracle baseline on a bounded sample of the same workload (rank 0, N = 1 only)
@@ -325,11 +369,12 @@ def main():
 
         sample = 1 << 27
         xs = x[:sample].cpu().numpy()
-        oracle.scan(xs[: 1 << 20], k, s, incl)
+        orun = (lambda a: oracle.delta(a, k, s)) if delta else (lambda a: oracle.scan(a, k, s, incl))
+        orun(xs[: 1 << 20])
         ts = []
         for _ in range(3):
             t0 = time.perf_counter()
-            oracle.scan(xs, k, s, incl)
+            orun(xs)
             ts.append(time.perf_counter() - t0)
         cpu = {"value": sample / statistics.median(ts) / 1e9, "unit": "Gvalues/s", "cores": 1, "kind": "oracle",
                "sample": f"first 2^27 elements of the same input, serial oracle (oracle/sam_oracle.c), median of 3"}
@@ -352,7 +397,7 @@ def main():
             "frac_of_memcpy": memcpy_ms / ms_per_step,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": ncu_traffic(args.config),
-                         "kernel": "sam::sam_scan_kernel", "kernel_ms": kavg,
+                         "kernel": "sam::delta_kernel" if delta else "sam::sam_scan_kernel", "kernel_ms": kavg,
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
             "cpu_baseline": cpu,
             "e2e": e2e,
