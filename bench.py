@@ -308,26 +308,29 @@ def main():
     if not args.no_e2e:
         xh = x.cpu().pin_memory()
         yh = torch.empty_like(xh).pin_memory()
-        if delta:
-            # encoder e2e: pinned H2D, sam_delta_encode (halo-exchanged under torchrun), D2H
+        if delta and world == 1:
+            sam.sam_delta_encode_host(dc, k, s, P(xh), P(yh), n_local, sp)
+            tt = []
+            for _ in range(3):
+                t0 = time.perf_counter()
+                sam.sam_delta_encode_host(dc, k, s, P(xh), P(yh), n_local, sp)
+                tt.append(time.perf_counter() - t0)
+            te = statistics.median(tt)
+        elif delta:
+            # encoder e2e under torchrun: pinned H2D, halo-exchanged encode, D2H
             xd = torch.empty_like(x)
             yd = torch.empty_like(x)
             tt = []
             for _ in range(4):
-                if world > 1:
-                    dist.barrier()
+                dist.barrier()
                 t0 = time.perf_counter()
                 xd.copy_(xh, non_blocking=True)
-                if world == 1:
-                    sam.sam_delta_encode(dc, k, s, P(xd), P(yd), n_local, sp)
-                else:
-                    delta_encode_sharded(xd, k, s, out=yd)
+                delta_encode_sharded(xd, k, s, out=yd)
                 yh.copy_(yd, non_blocking=True)
                 torch.cuda.synchronize()
                 tt.append(time.perf_counter() - t0)
             tte = torch.tensor([statistics.median(tt[1:])], dtype=torch.float64, device=dev)
-            if world > 1:
-                dist.all_reduce(tte, op=dist.ReduceOp.MAX)
+            dist.all_reduce(tte, op=dist.ReduceOp.MAX)
             te = float(tte[0])
             del xd, yd
         elif world == 1:
@@ -358,7 +361,8 @@ def main():
             te = float(tte[0])
         e2e = {"value": n_total / te / 1e9, "unit": "Gvalues/s", "h2d_bytes_per_step": n_local * w * world,
                "d2h_bytes_per_step": n_local * w * world, "ms_per_step": te * 1e3,
-               "path": "pinned H2D, sam_delta_encode, D2H (serial)" if delta else
+               "path": "sam_delta_encode_host: pinned host buffers, 128 MiB chunks, H2D | encode | D2H on 3 streams"
+               if delta and world == 1 else "per rank: pinned H2D, tail all-gather, encode, D2H" if delta else
                "sam_scan_host: pinned host buffers, 128 MiB chunks, H2D | seeded scan | D2H on 3 streams"
                if world == 1 else "per rank: pinned H2D, shard state, NCCL all-gather, shard scan, D2H"}
 

@@ -151,6 +151,13 @@ int sam_delta_encode(sam_dtype dtype, int order, int tuple, const void* in, void
 int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in, void* out, uint64_t n,
                           const void* halo, sam_stream_t stream);
 
+/* Host-buffer encoder (end-to-end path): like sam_scan_host, the array is streamed through the GPU
+ * in chunks, H2D | encode | D2H overlapping on separate streams; chunk j's halo is the last
+ * order*tuple inputs of chunk j-1 (kept on the device).  Synchronous.  in_host == out_host ->
+ * SAM_ERR_INVALID_ARG. */
+int sam_delta_encode_host(sam_dtype dtype, int order, int tuple, const void* in_host, void* out_host,
+                          uint64_t n, sam_stream_t stream);
+
 /* Diagnostics */
 const char* sam_last_error(void);
 const char* sam_version(void);

@@ -17,7 +17,7 @@ __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
     "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
-    "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
+    "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "sam_delta_encode_host", "delta_encode_host", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
 ]
 
 SAM_I32, SAM_I64, SAM_F32, SAM_F64 = 0, 1, 2, 3
@@ -55,6 +55,7 @@ def lib() -> ctypes.CDLL:
             "sam_fold_payloads_host": (I, [I, I, I, P, I, I, P]),
             "sam_delta_encode": (I, [I, I, I, P, P, U64, P]),
             "sam_delta_encode_halo": (I, [I, I, I, P, P, U64, P, P]),
+            "sam_delta_encode_host": (I, [I, I, I, P, P, U64, P]),
             "sam_last_error": (ctypes.c_char_p, []),
             "sam_version": (ctypes.c_char_p, []),
             "sam_release_workspaces": (I, []),
@@ -119,6 +120,10 @@ def sam_delta_encode(dtype, order, tuple_, in_ptr, out_ptr, n, stream=None) -> i
 
 def sam_delta_encode_halo(dtype, order, tuple_, in_ptr, out_ptr, n, halo_ptr, stream=None) -> int:
     return _check(lib().sam_delta_encode_halo(dtype, order, tuple_, in_ptr, out_ptr, n, halo_ptr, stream))
+
+
+def sam_delta_encode_host(dtype, order, tuple_, in_host_ptr, out_host_ptr, n, stream=None) -> int:
+    return _check(lib().sam_delta_encode_host(dtype, order, tuple_, in_host_ptr, out_host_ptr, n, stream))
 
 
 def sam_last_error() -> str:
@@ -188,6 +193,20 @@ def delta_encode(x, order: int = 1, tuple: int = 1, out=None, stream=None, halo=
         hp = None
     sam_delta_encode_halo(dtype_code(x.dtype), order, tuple, ctypes.c_void_p(x.data_ptr()),
                           ctypes.c_void_p(out.data_ptr()), x.numel(), hp, _stream_ptr(stream))
+    return out
+
+
+def delta_encode_host(x, order: int = 1, tuple: int = 1, out=None, stream=None):
+    """End-to-end delta encoding of a host (CPU) tensor through the GPU (sam_delta_encode_host:
+    chunked H2D | encode | D2H pipeline).  Pinned memory gives full PCIe bandwidth.  Synchronous."""
+    import torch
+
+    if x.is_cuda or x.dim() != 1 or not x.is_contiguous():
+        raise SamError(-1, "delta_encode_host() needs a 1-D contiguous CPU tensor")
+    if out is None:
+        out = torch.empty_like(x)
+    sam_delta_encode_host(dtype_code(x.dtype), order, tuple, ctypes.c_void_p(x.data_ptr()),
+                          ctypes.c_void_p(out.data_ptr()), x.numel(), _stream_ptr(stream))
     return out
 
 

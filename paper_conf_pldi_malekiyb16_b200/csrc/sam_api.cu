@@ -340,6 +340,8 @@ struct HostPipe {
     size_t chunk_bytes = 0;
     unsigned char* buf[NB] = {nullptr, nullptr, nullptr};
     unsigned char* state = nullptr;  // 2 x 512 B
+    unsigned char* obuf[NB] = {nullptr, nullptr, nullptr};  // encoder outputs (allocated on first use)
+    unsigned char* halo = nullptr;                         // encoder halos, 2 x 512 B
     cudaStream_t s_h2d = nullptr, s_cmp = nullptr, s_d2h = nullptr;
     cudaEvent_t ev_h2d[NB], ev_cmp[NB], ev_d2h[NB], ev_start;
 };
@@ -418,6 +420,67 @@ int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const vo
     cudaError_t e = cudaStreamSynchronize(P->s_d2h);
     if (e == cudaSuccess) e = cudaStreamSynchronize(P->s_cmp);
     if (e != cudaSuccess) return cuda_fail(e, "host pipeline");
+    return SAM_OK;
+}
+
+int sam_delta_encode_host(sam_dtype dtype, int order, int tuple, const void* in_host, void* out_host, uint64_t n,
+                          sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (n == 0) return SAM_OK;
+    if (!in_host || !out_host) return fail(SAM_ERR_INVALID_ARG, "null buffer with n > 0");
+    if (in_host == out_host) return fail(SAM_ERR_INVALID_ARG, "delta encoding is not done in place (P:281-284)");
+    std::lock_guard<std::mutex> lk(g_pipe_mu);
+    HostPipe* P = nullptr;
+    rc = get_pipe(&P);
+    if (rc) return rc;
+    if (!P->halo) {
+        for (int i = 0; i < HostPipe::NB; ++i)
+            if (cudaMalloc(&P->obuf[i], P->chunk_bytes) != cudaSuccess) return fail(SAM_ERR_OOM, "encoder buffers");
+        if (cudaMalloc(&P->halo, 1024) != cudaSuccess) return fail(SAM_ERR_OOM, "encoder halo");
+    }
+    const size_t w = elem_size(dtype);
+    const uint64_t C = P->chunk_bytes / w;  // >= order*tuple: only the last chunk is short
+    const uint64_t nchunks = (n + C - 1) / C;
+    const size_t hb = (size_t)order * tuple * w;
+    cudaStream_t user = (cudaStream_t)stream;
+    cudaEventRecord(P->ev_start, user);
+    cudaStreamWaitEvent(P->s_h2d, P->ev_start, 0);
+    cudaStreamWaitEvent(P->s_cmp, P->ev_start, 0);
+    cudaStreamWaitEvent(P->s_d2h, P->ev_start, 0);
+    for (uint64_t j = 0; j < nchunks; ++j) {
+        const int b = (int)(j % HostPipe::NB);
+        const uint64_t off = j * C;
+        const uint64_t cn = (n - off < C) ? n - off : C;
+        // buf[b] / obuf[b] are free once chunk j-NB has left the device
+        if (j >= (uint64_t)HostPipe::NB) {
+            cudaStreamWaitEvent(P->s_h2d, P->ev_d2h[b], 0);
+            cudaStreamWaitEvent(P->s_cmp, P->ev_d2h[b], 0);
+        }
+        cudaError_t e = cudaMemcpyAsync(P->buf[b], (const unsigned char*)in_host + off * w, cn * w,
+                                        cudaMemcpyHostToDevice, P->s_h2d);
+        if (e != cudaSuccess) return cuda_fail(e, "H2D");
+        cudaEventRecord(P->ev_h2d[b], P->s_h2d);
+        cudaStreamWaitEvent(P->s_cmp, P->ev_h2d[b], 0);
+        // chunk j's halo = the last order*tuple inputs of chunk j-1, saved on the compute stream
+        const void* halo = j ? (const void*)(P->halo + ((j - 1) & 1) * 512) : nullptr;
+        rc = sam_delta_encode_halo(dtype, order, tuple, P->buf[b], P->obuf[b], cn, halo, P->s_cmp);
+        if (rc) return rc;
+        if (j + 1 < nchunks) {
+            e = cudaMemcpyAsync(P->halo + (j & 1) * 512, P->buf[b] + cn * w - hb, hb, cudaMemcpyDeviceToDevice,
+                                P->s_cmp);
+            if (e != cudaSuccess) return cuda_fail(e, "halo copy");
+        }
+        cudaEventRecord(P->ev_cmp[b], P->s_cmp);
+        cudaStreamWaitEvent(P->s_d2h, P->ev_cmp[b], 0);
+        e = cudaMemcpyAsync((unsigned char*)out_host + off * w, P->obuf[b], cn * w, cudaMemcpyDeviceToHost,
+                            P->s_d2h);
+        if (e != cudaSuccess) return cuda_fail(e, "D2H");
+        cudaEventRecord(P->ev_d2h[b], P->s_d2h);
+    }
+    cudaError_t e = cudaStreamSynchronize(P->s_d2h);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(P->s_cmp);
+    if (e != cudaSuccess) return cuda_fail(e, "encoder host pipeline");
     return SAM_OK;
 }
 

@@ -155,3 +155,16 @@ def test_misaligned_output_scalar_path(name):
         y = S().delta_encode(xt, k, 1, out=buf[1:])
         torch.cuda.synchronize()
         check(name, x, y.cpu().numpy(), k, 1)
+
+
+@pytest.mark.parametrize("name,k,s,n", [("i32", 3, 5, (1 << 25) * 2 + 12345), ("i64", 8, 8, (1 << 24) + 777),
+                                        ("f32", 2, 1, 1000), ("i32", 1, 1, 1)])
+def test_host_pipeline(name, k, s, n):
+    # sam_delta_encode_host: chunks of 128 MiB (2^25 int32), halos carried across chunks on the device
+    x = synth.make_torch(n, name, "uniform", seed=k + s, device="cuda")
+    ref = S().delta_encode(x, k, s).cpu()
+    xh = x.cpu().pin_memory()
+    y = S().delta_encode_host(xh, k, s)
+    assert torch.equal(y.view(torch.uint8), ref.view(torch.uint8))
+    with pytest.raises(S().SamError):
+        S().delta_encode_host(xh, k, s, out=xh)
