@@ -80,6 +80,9 @@ def test_validation_invalid_args():
     assert L.sam_delta_encode(0, 9, 1, base, base + 256, 4, None) == -2         # order > 8
     assert L.sam_delta_encode(0, 1, 0, base, base + 256, 4, None) == -2         # tuple < 1
     assert L.sam_delta_encode(3, 1, 1, None, None, 0, None) == 0                # n == 0 is a no-op
+    assert L.sam_delta_encode_host(0, 2, 2, base, base, 4, None) == -1          # host encoder: not in place
+    assert L.sam_delta_encode_host(0, 0, 2, base, base + 256, 4, None) == -2    # order < 1
+    assert L.sam_delta_encode_host(0, 1, 1, None, None, 0, None) == 0           # n == 0 is a no-op
 
 
 @pytest.mark.parametrize("dt,k,s,expected", [(0, 1, 1, 32), (1, 4, 4, 144), (1, 8, 8, 528), (2, 3, 5, 80)])
