@@ -20,6 +20,7 @@
 // differencing bit for bit); fp32: accumulated in double, rounded once; fp64: accumulated in double.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 namespace sam {
 namespace {
@@ -27,6 +28,7 @@ namespace {
 constexpr int D_THREADS = 256;
 constexpr int D_HALO = 64;  // >= max k*s = 8*8
 constexpr int D_LANE_MIN_KS = 24;  // k*s from which s > 1 takes the lane-strided register path
+                                   // (SAM_DELTA_LANE_MIN_KS overrides: measurement knob)
 
 template <typename T> struct DeltaAcc { using type = T; };
 template <> struct DeltaAcc<float> { using type = double; };
@@ -43,7 +45,7 @@ template <typename T> __device__ __forceinline__ T zero_of() { return T(0); }
 template <typename T, int K>
 __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ in, T* __restrict__ out,
                                                            uint64_t n, int s, int vec_ok /* bit0 in, bit1 out 16-B aligned */,
-                                                           const T* __restrict__ halo) {
+                                                           const T* __restrict__ halo, int lane_min_ks) {
     using G = DeltaGeom<T>;
     using A = typename DeltaAcc<T>::type;
     __shared__ __align__(16) T sm[D_HALO + G::TILE];
@@ -115,7 +117,7 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
         return;
     }
 
-    if (s > 1 && ks >= D_LANE_MIN_KS) {
+    if (s > 1 && ks >= lane_min_ks) {
         // large k*s: lane-strided register path.  Unit u = (chunk c, lane m) owns the R positions
         // c*s*R + m + i*s (i < R) of one lane and keeps the K previous values of that lane in a
         // shift register, so a unit reads R + K smem values for R outputs instead of (K + 1) * R.
@@ -179,12 +181,20 @@ __global__ void __launch_bounds__(D_THREADS) delta_kernel(const T* __restrict__ 
     }
 }
 
+int lane_min_ks() {
+    static const int v = [] {
+        const char* e = getenv("SAM_DELTA_LANE_MIN_KS");
+        return e ? atoi(e) : D_LANE_MIN_KS;
+    }();
+    return v;
+}
+
 template <typename T, int K>
 cudaError_t launch_k(const T* in, T* out, uint64_t n, int s, const T* halo, cudaStream_t st) {
     using G = DeltaGeom<T>;
     const uint64_t tiles = (n + G::TILE - 1) / G::TILE;
     const int vec_ok = (((uintptr_t)in % 16) == 0 ? 1 : 0) | (((uintptr_t)out % 16) == 0 ? 2 : 0);
-    delta_kernel<T, K><<<(unsigned)tiles, D_THREADS, 0, st>>>(in, out, n, s, vec_ok, halo);
+    delta_kernel<T, K><<<(unsigned)tiles, D_THREADS, 0, st>>>(in, out, n, s, vec_ok, halo, lane_min_ks());
     return cudaGetLastError();
 }
 
