@@ -21,13 +21,24 @@
  * MEMORY AND OWNERSHIP
  *   `in`, `out`, payload buffers: device pointers (cudaMalloc / torch CUDA tensors) on the
  *   current device, owned by the caller, aligned to the element size.  `in == out` (in-place)
- *   is allowed; any other overlap is SAM_ERR_INVALID_ARG.  The library owns only a workspace
- *   (tile status/state arrays, a few counters) cached per (device, stream), grown lazily and
- *   kept for the life of the process (sam_release_workspaces frees it).  Calls on one stream
- *   are ordered; calls on different streams use different workspaces and may run concurrently.
- *   CUDA-graph capture is supported (the kernel resets its counters itself, no host state
- *   changes between replays) provided the workspace was created before capture (make one
- *   un-captured call, or call sam_prepare).
+ *   is allowed; any other overlap is SAM_ERR_INVALID_ARG.  Scratch (epoch-tagged carry words,
+ *   a few counters) lives either in a workspace the library caches per (device, stream), grown
+ *   lazily -- growing synchronises the stream -- and kept for the life of the process
+ *   (sam_release_workspaces frees it), or, with sam_scan_ws, in a caller-owned workspace
+ *   (no allocation, no synchronisation: the form for graph capture and concurrent streams).
+ *   Calls on one stream are ordered; calls on different streams use different workspaces and
+ *   may run concurrently.  The kernel resets its own counters and validates carry words by a
+ *   per-launch epoch tag, so CUDA-graph replays need no host work (with the cached workspace,
+ *   create it before capture: one un-captured call, or sam_prepare).
+ *
+ * EXECUTION MODEL
+ *   One kernel launch per scan: a persistent grid of P co-resident CTAs (one per SM, launched
+ *   cooperatively) runs SAM's static carry schedule: CTA b owns super-tiles b,
+ *   b+P, b+2P, ...; the carry into super-tile S is the CTA's own inclusive state after S-P
+ *   combined with the aggregates the other P-1 CTAs published in between.  This needs all P
+ *   CTAs resident at once.  If the driver refuses the cooperative grid (MPS SM limits, a green
+ *   context, an SM-partitioned device), the launch retries with a smaller grid -- the schedule
+ *   is correct for any P -- and the reduced size is remembered for the device.
  *
  * ERRORS
  *   Every entry point returns a sam_status.  Argument validation happens synchronously before
@@ -62,7 +73,8 @@ typedef void* sam_stream_t;
 /*
  * sam_scan -- single-GPU order-k, tuple-s, inclusive/exclusive scan of n scalars.
  * One kernel launch, one read of `in` and one write of `out`, the
- * inter-tile carries propagated by decoupled look-back.
+ * inter-tile carries propagated by SAM's static persistent-block schedule (see
+ * EXECUTION MODEL above).
  *   dtype      element type of in/out (n elements each)
  *   order      k, 1..8          tuple  s, 1..8          inclusive  nonzero = inclusive
  *   n          number of scalars (not tuples); n = 0 is a no-op returning SAM_OK
@@ -88,6 +100,24 @@ int sam_scan_seeded(sam_dtype dtype, int order, int tuple, int inclusive, const 
 /* Make sure the workspace for (current device, stream) exists (optional; useful before graph
  * capture).  `max_n` sizes it for streams of up to max_n elements. */
 int sam_prepare(sam_dtype dtype, int order, int tuple, uint64_t max_n, sam_stream_t stream);
+
+/*
+ * Explicit-workspace form (CUB-style), for graph capture and concurrent streams: no allocation,
+ * no synchronisation, no library state per stream.
+ *   sam_scan_workspace_size  *bytes = workspace bytes sam_scan_ws needs for (dtype, order, tuple,
+ *                            n); a workspace sized for n serves any n' <= n.
+ *   sam_scan_ws              sam_scan with the caller's workspace `ws` (device memory, 16-B
+ *                            aligned, ws_bytes >= the size above).  The caller ZERO-FILLS the
+ *                            workspace once before its first use (cudaMemsetAsync); afterwards the
+ *                            kernel maintains it (epoch tags, counters reset by the last CTA of
+ *                            each launch, a full reset when the 32-bit epoch wraps).  One
+ *                            workspace serves one scan at a time: calls ordered on one stream may
+ *                            share it, concurrent calls need distinct workspaces.
+ *   Errors: as sam_scan; null/misaligned ws or ws_bytes too small -> SAM_ERR_INVALID_ARG.
+ */
+int sam_scan_workspace_size(sam_dtype dtype, int order, int tuple, uint64_t n, size_t* bytes);
+int sam_scan_ws(sam_dtype dtype, int order, int tuple, int inclusive, const void* in, void* out,
+                uint64_t n, void* ws, size_t ws_bytes, sam_stream_t stream);
 
 /*
  * Host-buffer entry point (end-to-end path): `in_host` / `out_host` are host pointers
@@ -164,6 +194,13 @@ const char* sam_version(void);
 int sam_release_workspaces(void);
 /* Kernel launches issued by this library on the calling process since load (for bench). */
 uint64_t sam_launch_count(void);
+/* Testing: treat persistent grids above max_ctas CTAs as refused by the driver (0 = off), so the
+ * cooperative-launch fallback shrinks the grid (to <= max_ctas) exactly as it does under MPS. */
+int sam_debug_limit_grid(uint64_t max_ctas);
+/* Testing: nonzero seed = pseudo-random delays (up to ~16 us, 1 in 8 events) at every pipeline
+ * hand-over of subsequent scan launches (loads, aggregate publication, carry folds, hand-offs,
+ * local scans, carry applications), so the warps and CTAs meet in shuffled orders; 0 = off. */
+int sam_debug_set_stress(uint32_t seed);
 /* Diagnostics: when trace_dev (device memory, >= 16 * tiles u64, zeroed) is non-NULL, subsequent
  * scan launches record %globaltimer at pipeline events of every tile: [tile][claim, P1 start,
  * P1 done, aggregate published, look-back start, inclusive published, carry applied, stored,

@@ -15,7 +15,8 @@ import os
 
 __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
-    "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_shard_payload_bytes",
+    "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_scan_workspace_size", "sam_scan_ws",
+    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
     "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "sam_delta_encode_host", "delta_encode_host", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
 ]
@@ -61,6 +62,10 @@ def lib() -> ctypes.CDLL:
             "sam_release_workspaces": (I, []),
             "sam_launch_count": (U64, []),
             "sam_debug_set_trace": (I, [P]),
+            "sam_debug_limit_grid": (I, [U64]),
+            "sam_debug_set_stress": (I, [ctypes.c_uint32]),
+            "sam_scan_workspace_size": (I, [I, I, I, U64, ctypes.POINTER(SZ)]),
+            "sam_scan_ws": (I, [I, I, I, I, P, P, U64, P, SZ, P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -90,6 +95,25 @@ def sam_scan_seeded(dtype, order, tuple_, inclusive, in_ptr, out_ptr, n, global_
 def sam_scan_host(dtype, order, tuple_, inclusive, in_host_ptr, out_host_ptr, n, stream=None) -> int:
     return _check(lib().sam_scan_host(dtype, order, tuple_, int(bool(inclusive)), in_host_ptr, out_host_ptr, n,
                                       stream))
+
+
+def sam_scan_workspace_size(dtype, order, tuple_, n) -> int:
+    b = ctypes.c_size_t(0)
+    _check(lib().sam_scan_workspace_size(dtype, order, tuple_, n, ctypes.byref(b)))
+    return int(b.value)
+
+
+def sam_scan_ws(dtype, order, tuple_, inclusive, in_ptr, out_ptr, n, ws_ptr, ws_bytes, stream=None) -> int:
+    return _check(lib().sam_scan_ws(dtype, order, tuple_, int(bool(inclusive)), in_ptr, out_ptr, n, ws_ptr,
+                                    ws_bytes, stream))
+
+
+def sam_debug_limit_grid(max_ctas: int) -> int:
+    return _check(lib().sam_debug_limit_grid(max_ctas))
+
+
+def sam_debug_set_stress(seed: int) -> int:
+    return _check(lib().sam_debug_set_stress(seed))
 
 
 def sam_prepare(dtype, order, tuple_, max_n, stream=None) -> int:

@@ -28,7 +28,7 @@ namespace {
 
 thread_local std::string g_err;
 std::atomic<uint64_t> g_launches{0};
-constexpr const char* kVersion = "sam-b200 0.1 (sm_100a, single-pass decoupled look-back, order 1-8, tuple 1-8)";
+constexpr const char* kVersion = "sam-b200 0.2 (sm_100a, single-pass, SAM static carry schedule on a cooperative persistent grid, order 1-8, tuple 1-8)";
 
 int fail(int code, const std::string& msg) {
     g_err = msg;
@@ -96,7 +96,10 @@ int num_sms(int dev) {
     return n;
 }
 
+// Workspace header (device memory): [u64 tile_ctr][u32 done][u32 epoch][u32 reset][pad .. 32]
+// [512 B seed scratch of sam_shard_scan][pad .. 1024], then the tagged carry words.
 constexpr size_t CTR_BYTES = 32 + 8 * 8 * 8;
+constexpr size_t WS_HEADER = 1024;
 
 // workspace of (current device, stream) with room for `carry_bytes` of tagged carry words
 int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out) {
@@ -114,6 +117,7 @@ int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out) {
     }
     if (carry_bytes > ws->carry_cap) {
         // grow (never shrink); the old buffer may still be read by queued kernels on this stream
+        // (graph capture / concurrent streams: use sam_scan_ws with a caller-owned workspace)
         e = cudaStreamSynchronize(st);
         if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
         const size_t cap = carry_bytes + carry_bytes / 4 + 4096;
@@ -141,9 +145,14 @@ int items_of(sam_dtype d) {
     }
 }
 
-// bytes of tagged carry words for `tiles` tiles: per (lane, order) 2 values x (1 or 2) words
+// bytes of tagged carry words for `tiles` tiles (an upper bound of the super-tiles): per (super-tile,
+// lane, order) one value in 1 (4-byte types) or 2 (8-byte types) 64-bit words
 size_t carry_bytes(sam_dtype d, int k, int s, size_t tiles) {
-    return tiles * (size_t)s * (size_t)k * 2 * (elem_size(d) / 4) * 8;
+    return tiles * (size_t)s * (size_t)k * (elem_size(d) / 4) * 8;
+}
+size_t tiles_for(sam_dtype dtype, int s, uint64_t n) {
+    const sam::Geom geo = sam::make_geom(s, items_of(dtype));
+    return (size_t)((n + (uint64_t)s + geo.T - 1) / geo.T);
 }
 
 template <typename T>
@@ -164,16 +173,23 @@ cudaError_t dispatch_k(int k, const sam::LaunchArgs& a) {
     return e;
 }
 
-// one scan-kernel launch for a stream of n elements at global offset g
+// one scan-kernel launch for a stream of n elements at global offset g.  ws_hdr / carry / carry_cap:
+// an explicit workspace (sam_scan_ws), or null for the cached (device, stream) workspace.
 int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void* out, uint64_t n, uint64_t g,
-             const void* seed, void* final_state, int store_mode, cudaStream_t st) {
-    const sam::Geom geo = sam::make_geom(s, items_of(dtype));
-    const uint64_t h = g % (uint64_t)s;
-    const size_t tiles = (size_t)((h + n + geo.T - 1) / geo.T);
-    Workspace* ws = nullptr;
+             const void* seed, void* final_state, int store_mode, cudaStream_t st,
+             unsigned char* ws_hdr = nullptr, unsigned long long* ws_carry = nullptr, size_t ws_carry_cap = 0) {
     int dev = 0;
-    int rc = get_ws(st, carry_bytes(dtype, k, s, tiles), &ws, &dev);
-    if (rc != SAM_OK) return rc;
+    if (!ws_hdr) {
+        Workspace* ws = nullptr;
+        int rc = get_ws(st, carry_bytes(dtype, k, s, tiles_for(dtype, s, n + g % (uint64_t)s)), &ws, &dev);
+        if (rc != SAM_OK) return rc;
+        ws_hdr = ws->ctr;
+        ws_carry = ws->carry;
+        ws_carry_cap = ws->carry_cap;
+    } else {
+        cudaError_t e = cudaGetDevice(&dev);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    }
     sam::LaunchArgs a;
     a.in = in;
     a.out = out;
@@ -185,11 +201,14 @@ int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void*
     a.inclusive = inclusive ? 1 : 0;
     a.store_mode = store_mode;
     a.stream = st;
-    a.carry = ws->carry;
-    a.tile_ctr = (unsigned long long*)(ws->ctr);
-    a.done_ctr = (unsigned int*)(ws->ctr + 8);
-    a.epoch_ptr = (unsigned int*)(ws->ctr + 12);
+    a.carry = ws_carry;
+    a.carry_words = ws_carry_cap / 8;
+    a.tile_ctr = (unsigned long long*)(ws_hdr);
+    a.done_ctr = (unsigned int*)(ws_hdr + 8);
+    a.epoch_ptr = (unsigned int*)(ws_hdr + 12);
+    a.reset_ctr = (unsigned int*)(ws_hdr + 16);
     a.num_sms = num_sms(dev);
+    a.dev = dev;
     a.trace = g_trace;
     cudaError_t e;
     switch (dtype) {
@@ -248,11 +267,35 @@ int sam_scan_seeded(sam_dtype dtype, int order, int tuple, int inclusive, const 
 int sam_prepare(sam_dtype dtype, int order, int tuple, uint64_t max_n, sam_stream_t stream) {
     int rc = validate_common(dtype, order, tuple);
     if (rc) return rc;
-    const sam::Geom geo = sam::make_geom(tuple, items_of(dtype));
-    const size_t tiles = (size_t)((max_n + tuple + geo.T - 1) / geo.T);
     Workspace* ws = nullptr;
     int dev = 0;
-    return get_ws((cudaStream_t)stream, carry_bytes(dtype, order, tuple, tiles), &ws, &dev);
+    return get_ws((cudaStream_t)stream, carry_bytes(dtype, order, tuple, tiles_for(dtype, tuple, max_n)), &ws, &dev);
+}
+
+int sam_scan_workspace_size(sam_dtype dtype, int order, int tuple, uint64_t n, size_t* bytes) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (!bytes) return fail(SAM_ERR_INVALID_ARG, "null bytes pointer");
+    *bytes = WS_HEADER + carry_bytes(dtype, order, tuple, tiles_for(dtype, tuple, n));
+    return SAM_OK;
+}
+
+int sam_scan_ws(sam_dtype dtype, int order, int tuple, int inclusive, const void* in, void* out, uint64_t n,
+                void* ws, size_t ws_bytes, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    rc = validate_buffers(dtype, in, out, n, true);
+    if (rc) return rc;
+    if (n == 0) return SAM_OK;
+    size_t need = 0;
+    sam_scan_workspace_size(dtype, order, tuple, n, &need);
+    if (!ws) return fail(SAM_ERR_INVALID_ARG, "null workspace");
+    if (((uintptr_t)ws & 15) != 0) return fail(SAM_ERR_INVALID_ARG, "workspace must be 16-B aligned");
+    if (ws_bytes < need)
+        return fail(SAM_ERR_INVALID_ARG, "workspace too small (sam_scan_workspace_size gives " + std::to_string(need) + " B)");
+    unsigned char* w = (unsigned char*)ws;
+    return run_scan(dtype, order, tuple, inclusive, in, out, n, 0, nullptr, nullptr, store_mode_for(in, out),
+                    (cudaStream_t)stream, w, (unsigned long long*)(w + WS_HEADER), ws_bytes - WS_HEADER);
 }
 
 size_t sam_shard_payload_bytes(sam_dtype dtype, int order, int tuple) {
@@ -511,6 +554,17 @@ int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in,
     }
     g_launches += l;
     return e == cudaSuccess ? SAM_OK : cuda_fail(e, "delta encoder launch");
+}
+
+int sam_debug_limit_grid(uint64_t max_ctas) {
+    sam::debug_grid_limit() = max_ctas;
+    for (int d = 0; d < sam::MAX_DEVICES; ++d) sam::debug_grid_cap(d) = 0;
+    return SAM_OK;
+}
+
+int sam_debug_set_stress(uint32_t seed) {
+    sam::debug_stress() = seed;
+    return SAM_OK;
 }
 
 int sam_debug_set_trace(void* trace_dev) {

@@ -5,15 +5,14 @@
 // tuple size.  Persistent, warp-specialised CTAs (one per SM) stream tiles of
 // T = W*32*ITEMS elements:
 //
-//   producer warp   a1: claims tiles from an atomic counter, one at a time and at most PF ahead
-//                   of the local scans (every predecessor of a claimed tile belongs to a running
-//                   CTA -- no co-residency assumption), and pulls each tile
-//                   from HBM into a ring of NB1 smem buffers with a 1-D cp.async.bulk (TMA bulk
-//                   engine) marked L2::evict_last.  When the tile's carry is known it pulls the
-//                   same bytes again -- now from the 126 MB L2 (~18 TB/s vs ~7 TB/s HBM) -- into a
-//                   second ring of NB2 buffers, and a7: writes the finished tile back with a
-//                   cp.async.bulk store.  The look-back's latency is spent with the tile parked
-//                   in L2, not in shared memory, so it no longer throttles the HBM stream.
+//   producer warp   a1: walks this CTA's static schedule (super-tiles b, b+P, b+2P, ..., P = the
+//                   co-resident grid of a cooperative launch) at most PF tiles ahead of the local
+//                   scans, and pulls each tile from HBM into a ring of NB1 smem buffers with a 1-D
+//                   cp.async.bulk (TMA bulk engine) marked L2::evict_last.  When the tile's carry
+//                   is known it pulls the same bytes again -- now from the 126 MB L2 (~18 TB/s vs
+//                   ~7 TB/s HBM) -- into a second ring of NB2 buffers, and a7: writes the finished
+//                   tile back with a cp.async.bulk store.  The carry's latency is spent with the
+//                   tile parked in L2, not in shared memory, so it does not throttle the stream.
 //   compute warps   a2: thread <-> (tuple lane m, ITEMS consecutive lane positions), read from
 //                   smem at stride s; a warp holds G = (largest power of two dividing s) lanes,
 //                   32/G threads each, so the strided reads are bank-conflict free (ITEMS odd)
@@ -30,14 +29,15 @@
 //                   CTAs' look-backs); up to LAG tiles may await their carries.
 //   aggregator warp a3/a4: combines the warp states of a tile and publishes its per-lane k-vector
 //                   aggregate (one value per order; all s lanes).
-//   carry warps     a5: decoupled look-back.  Every published 64-bit word carries the launch's
+//   carry warps     a5: SAM's carry scheme on a static schedule: the carry into
+//                   super-tile S is this CTA's own inclusive state after S-P (handed over in
+//                   shared memory) advanced over the P-1 aggregates the other CTAs published in
+//                   between, read in windows (one L2 round trip each) and folded with the carry
+//                   operator (M(L) s + v).  Every published 64-bit word carries the launch's
 //                   32-bit epoch tag beside (half) a value, so each word validates itself: the
-//                   paper's "local sum -> fence -> ready flag" becomes one store with
-//                   no fence, and a look-back hop is ONE L2 round trip over a window of up to 512
-//                   predecessor tiles, folded with the carry operator (M(L) s + v) back to the
-//                   nearest inclusive state -- the O(n) scheme the paper describes for CUB
-//                    and advises once the architectural factor grows (
-//                   B200's af is ~9x the paper's GPUs).
+//                   paper's "local sum -> fence -> ready flag" becomes one store
+//                   with no fence.  All P CTAs must be co-resident (cooperative launch); there
+//                   is no inclusive chain between CTAs, only between a CTA's own super-tiles.
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -201,7 +201,10 @@ struct Params {
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
+    unsigned long long carry_words;  // capacity of `carry` (64-bit words)
+    unsigned int* reset_ctr;         // grid barrier of the epoch wrap-around reset
     unsigned long long* trace;  // optional per-tile event timestamps [tile][8] (diagnostics), or null
+    uint32_t stress;            // testing: nonzero = seed of pseudo-random delays at every pipeline hand-over
     T bc[K];              // b_d(ITEMS)
     T bw[K];              // b_d(Uw)
     T bu[K];              // b_d(U)        (one tile)
@@ -298,6 +301,20 @@ __device__ __forceinline__ unsigned long long globaltimer() {
 #define SAM_TRACE(ev, tile)                                                        \
     do {                                                                           \
         if (p.trace) p.trace[(size_t)(tile) * 16 + (ev)] = globaltimer();          \
+    } while (0)
+// testing (sam_debug_set_stress): a pseudo-random delay of up to ~16 us at 1 in 8 of the
+// pipeline events, so the hand-overs between warps and CTAs happen in shuffled orders
+static __device__ __noinline__ void stress_delay(uint32_t seed, uint64_t tile, uint32_t ev) {
+    uint64_t h = tile * 0x9E3779B97F4A7C15ull ^ (uint64_t)(ev + 1) * 0xC2B2AE3D27D4EB4Full ^ seed;
+    h ^= h >> 29;
+    h *= 0xBF58476D1CE4E5B9ull;
+    h ^= h >> 32;
+    const uint32_t r = (uint32_t)h;
+    if ((r & 7) == 0) __nanosleep((r >> 8) & 16383);
+}
+#define SAM_STRESS(ev, tile)                                                       \
+    do {                                                                           \
+        if (p.stress) stress_delay(p.stress, (uint64_t)(tile), (ev));              \
     } while (0)
 __device__ __forceinline__ uint64_t policy_evict_last() {
     uint64_t p;
@@ -479,7 +496,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             *(volatile int*)(smem + S::OFF_HO + w * S::HOB) = -1;
         }
         fence_mbar_init();
-        *sm_tag = *(volatile unsigned int*)p.epoch_ptr + 1u;  // tags are never 0 (zeroed workspace)
+        // tags are never 0 (zero-filled workspace); when the 32-bit epoch wraps, this launch first
+        // zeroes every carry word (below) so no word tagged 2^32 launches ago can validate
+        const unsigned ep = *(volatile unsigned int*)p.epoch_ptr;
+        *sm_tag = ep == 0xffffffffu ? 0u : ep + 1u;
         *sm_end = -1;
         *agg_done = 0;
         *(volatile int*)(smem + S::OFF_TAG + 12) = 0;
@@ -489,6 +509,21 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
     for (int i = tid; i < 8 * K; i += blockDim.x) bq_s[i] = (&p.bq[0][0])[i];
     __syncthreads();
+    if (*sm_tag == 0u) {  // epoch wrap-around (once per 2^32 launches of a workspace)
+        for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + tid; i < p.carry_words;
+             i += (unsigned long long)gridDim.x * blockDim.x)
+            p.carry[i] = 0ull;
+        __syncthreads();
+        if (tid == 0) {  // grid barrier (all CTAs co-resident: cooperative launch)
+            __threadfence();
+            atomicAdd(p.reset_ctr, 1u);
+            while (*(volatile unsigned int*)p.reset_ctr < gridDim.x) __nanosleep(100);
+            __threadfence();
+            *sm_tag = 1u;
+            if (blockIdx.x == 0) *(volatile unsigned int*)p.epoch_ptr = 0u;  // the epilogue makes it 1
+        }
+        __syncthreads();
+    }
     const uint32_t tag = *sm_tag;
 
     // wait for barrier phase `par`, or return false once the stream has ended before iteration it
@@ -594,6 +629,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         sub_of[2 * qs + 1] = cur_cnt;
                         ++cur_j;
                         SAM_TRACE(0, t);
+                        SAM_STRESS(0, t);
                         load_tile(t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1], pol_keep);
                         ++j1;
                     }
@@ -619,6 +655,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const int64_t sup = sup_of[qs];
             const int jsub = sub_of[2 * qs], cnt = sub_of[2 * qs + 1];
             if (lane == 0) SAM_TRACE(2, tile);
+            SAM_STRESS(1, tile);
             T* wq = wq_all + qs * S::WQ;
             T* la = la_all + qs * S::LA;
             T* lp = lp_all + qs * S::LA;
@@ -760,6 +797,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 if (SAM_EARLY_RELOAD == 2) *lb_started = r;  // its tiles may be re-fetched from L2 now
             }
 
+            SAM_STRESS(2 + cw, tile);
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, T* out) {
                 if (p.seed) {
@@ -990,6 +1028,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
             }
             if (lane == 0) SAM_TRACE(14, tile * p.M);
+            SAM_STRESS(6, tile);
             // each sub-tile j: C_j = M(j U) C + P_j, then per-warp incoming states
             // C_{m,q} = M(q*Uw) C_{j,m} + E_{m,q}  (E in wq, from the combine)
             for (int j = 0; j < cnt; ++j) {
@@ -1045,6 +1084,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const int b2 = it % NB2;
             const int qs = it % NQ;
             if (gtid == 0) SAM_TRACE(6, tile);
+            SAM_STRESS(8 + warp, tile);
             T* xs = (T*)(smem + S::OFF_BUF2 + b2 * S::BUFB + p.delta);
             const T* wq = wq_all + qs * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
@@ -1209,6 +1249,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const int qs = i % NQ;
             const int64_t tile = tile_of[qs];
             if (gtid == 0) SAM_TRACE(1, tile);
+            SAM_STRESS(32 + warp, tile);
             const T* xs = (const T*)(smem + S::OFF_BUF1 + b1 * S::BUFB + p.delta);
             T* wq = wq_all + qs * S::WQ;
             const uint64_t e0 = (uint64_t)tile * (uint64_t)Tt;
@@ -1416,6 +1457,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         if (prev == gridDim.x - 1) {
             *(volatile unsigned long long*)p.tile_ctr = 0ull;
             *(volatile unsigned int*)p.done_ctr = 0u;
+            *(volatile unsigned int*)p.reset_ctr = 0u;
             __threadfence();
             atomicAdd(p.epoch_ptr, 1u);
         }

@@ -6,6 +6,7 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include <map>
 #include <mutex>
 
 #include "sam_algebra.h"
@@ -62,17 +63,61 @@ struct LaunchArgs {
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
     unsigned long long* trace;
+    unsigned long long carry_words;  // capacity of `carry` in 64-bit words (wrap-around reset)
+    unsigned int* reset_ctr;         // grid barrier of the epoch wrap-around reset
     int num_sms;
+    int dev;
 };
 
 template <typename T>
 inline int items_of() { return Cfg<T>::ITEMS; }
 
+// Experiment knobs (developer tools only), read from the environment ONCE per process -- never on
+// the per-launch path.  0 / -1 = unset.
+struct Knobs {
+    int claim_slack = 0;   // SAM_CLAIM_SLACK: extra claimed-but-blocked tiles (ring slots allow <= 2)
+    int super_tile = 0;    // SAM_SUPER_TILE: force the tiles per super-tile (1..8)
+    int vr = 0;            // SAM_VR: window rows per round trip
+    int coop = -1;         // SAM_COOP: carry warps fold each super-tile together (1) or round-robin (0)
+    bool no_vec = false;   // SAM_NO_VEC: never take the 128-bit tuple-1 path
+};
+inline const Knobs& knobs() {
+    static const Knobs k = [] {
+        Knobs r;
+        if (const char* e = getenv("SAM_CLAIM_SLACK")) { const int v = atoi(e); r.claim_slack = v < 0 ? 0 : (v > 2 ? 2 : v); }
+        if (const char* e = getenv("SAM_SUPER_TILE")) { const int v = atoi(e); if (v >= 1 && v <= 8) r.super_tile = v; }
+        if (const char* e = getenv("SAM_VR")) r.vr = atoi(e);
+        if (const char* e = getenv("SAM_COOP")) r.coop = atoi(e) != 0;
+        r.no_vec = getenv("SAM_NO_VEC") != nullptr;
+        return r;
+    }();
+    return k;
+}
+
+constexpr int MAX_DEVICES = 64;
+
+// Per-device launch facts of one kernel instantiation: the dynamic-shared-memory opt-in
+// (cudaFuncSetAttribute is per device context) and the occupancy, set on first use on each device.
 template <typename T, int K, bool VEC>
 struct KernelInfo {
-    int max_blocks_per_sm = 0;
-    bool ready = false;
+    int max_blocks_per_sm[MAX_DEVICES] = {};
+    bool ready[MAX_DEVICES] = {};
     std::mutex mu;
+};
+
+// Host-side tables of a launch shape (the binomial columns b_d(L) of every span the kernel combines
+// over: ~300 exact 128-bit evaluations), cached per (device, s, M, P, Vr) so a launch only fills in
+// its per-call fields.
+struct ShapeKey {
+    int dev, s, M, Vr;
+    uint64_t P;
+    bool operator<(const ShapeKey& o) const {
+        if (dev != o.dev) return dev < o.dev;
+        if (s != o.s) return s < o.s;
+        if (M != o.M) return M < o.M;
+        if (Vr != o.Vr) return Vr < o.Vr;
+        return P < o.P;
+    }
 };
 
 // persistent grid: all co-resident CTAs, at most one per super-tile
@@ -82,137 +127,178 @@ inline uint64_t grid_of(int blocks_per_sm, int num_sms, uint64_t num_super) {
     return grid < 1 ? 1 : grid;
 }
 
+// cooperative-grid cap per device (debug: sam_debug_limit_grid; the fallback lowers it when the
+// driver refuses a cooperative grid, e.g. under MPS SM limits or in a green context)
+inline uint64_t& grid_cap(int dev) {
+    static uint64_t cap[MAX_DEVICES] = {};
+    return cap[dev];
+}
+// testing (sam_debug_limit_grid): grids above the limit are treated as refused by the driver, so
+// the shrink-and-retry path runs; what it learns is kept apart from grid_cap and reset with the limit
+inline uint64_t& debug_grid_limit() {
+    static uint64_t lim = 0;
+    return lim;
+}
+inline uint64_t& debug_grid_cap(int dev) {
+    static uint64_t cap[MAX_DEVICES] = {};
+    return cap[dev];
+}
+inline uint32_t& debug_stress() {
+    static uint32_t seed = 0;
+    return seed;
+}
+
 template <typename T, int K, bool VEC>
 cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
     using S = Smem<T, K, VEC>;
     constexpr int ITEMS = Items<T, VEC>::V;
+    constexpr int V = LB<T, K>::V;
     static KernelInfo<T, K, VEC> info;
+    static std::map<ShapeKey, Params<T, K>*> tables;  // guarded by info.mu
+    const Knobs& kn = knobs();
+    const int dev = a.dev;
+    if (dev < 0 || dev >= MAX_DEVICES) return cudaErrorInvalidDevice;
+    int maxb;
     {
         std::lock_guard<std::mutex> lk(info.mu);
-        if (!info.ready) {
+        if (!info.ready[dev]) {
             cudaError_t e = cudaFuncSetAttribute(sam_scan_kernel<T, K, VEC>,
                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES);
             if (e != cudaSuccess) return e;
             int nb = 0;
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K, VEC>, Threads<T, K>::VALUE, S::BYTES);
             if (e != cudaSuccess) return e;
-            info.max_blocks_per_sm = nb > 0 ? nb : 1;
-            info.ready = true;
+            info.max_blocks_per_sm[dev] = nb > 0 ? nb : 1;
+            info.ready[dev] = true;
         }
+        maxb = info.max_blocks_per_sm[dev];
     }
     const Geom geo = make_geom(a.s, ITEMS);
-    Params<T, K> p;
-    memset(&p, 0, sizeof(p));
-    p.in = (const T*)a.in;
-    p.out = (T*)a.out;
-    p.n = a.n;
-    p.h = a.g % (uint64_t)a.s;
-    p.num_tiles = (p.h + a.n + geo.T - 1) / geo.T;
-    p.delta = (uint32_t)(((uintptr_t)a.in - p.h * sizeof(T)) & 15);
-    p.s = geo.s; p.G = geo.G; p.logG = geo.logG; p.sp = geo.sp; p.c = geo.c; p.logc = geo.logc;
-    p.Pw = geo.Pw; p.W = geo.W; p.Wn = geo.Wn; p.U = geo.U; p.T_ = geo.T; p.Uw = geo.Uw;
-    p.inclusive = a.inclusive;
-    p.store_mode = a.store_mode;
-    if (const char* env = getenv("SAM_CLAIM_SLACK")) {  // experiments (ring slots allow at most 2)
-        const int v = atoi(env);
-        p.claim_slack = v < 0 ? 0 : (v > 2 ? 2 : v);
-    }
-    p.seed = (const T*)a.seed;
-    p.final_state = (T*)a.final_state;
-    for (int m = 0; m < MAXS; ++m) {
-        p.last_e[m] = -1;
-        if (m < a.s && a.n > 0) {
-            const int64_t eend = (int64_t)(p.h + a.n - 1);
-            const int64_t le = eend - ((eend - m) % a.s + a.s) % a.s;
-            if (le >= (int64_t)p.h && le >= 0) p.last_e[m] = le;
-        }
-    }
-    p.carry = a.carry;
-    p.tile_ctr = a.tile_ctr;
-    p.done_ctr = a.done_ctr;
-    p.epoch_ptr = a.epoch_ptr;
-    p.trace = a.trace;
-    // super-tile size: up to MMAX tiles per look-back unit, but keep >= 2 super-tiles per SM
+    const uint64_t h = a.g % (uint64_t)a.s;
+    const uint64_t num_tiles = (h + a.n + geo.T - 1) / geo.T;
+    // super-tile size: up to MMAX tiles per carry unit, but keep >= 2 super-tiles per SM
+    uint64_t M;
     {
-        uint64_t m = p.num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
-        if (m < 1) m = 1;
+        M = num_tiles / (2ull * (uint64_t)(a.num_sms > 0 ? a.num_sms : 148));
+        if (M < 1) M = 1;
         // measured: tuple 1: 3 (4-byte) / 2 (8-byte) tiles; tuples (more carry-team work per unit):
         // 3, or 4 for odd tuples of 4-byte elements (~1.5% better there)
         const uint64_t mmax = a.s == 1 ? (uint64_t)Lag<T, K>::MMAX : ((sizeof(T) == 4 && (a.s & 1)) ? 4u : 3u);
-        if (m > mmax) m = mmax;
-        if (const char* env = getenv("SAM_SUPER_TILE")) {  // experiments: force a smaller super-tile
-            const int f = atoi(env);
-            if (f >= 1 && f <= 8) m = (uint64_t)f;
-        }
+        if (M > mmax) M = mmax;
+        if (kn.super_tile) M = (uint64_t)kn.super_tile;
         // a super-tile is aggregated before its carry is known: at most LAG/2 tiles per unit
         // keep two units in flight per CTA (LAG bounds the tiles between load and carry application)
         const uint64_t mlag = Lag<T, K>::LAG / 2 > 1 ? Lag<T, K>::LAG / 2 : 1;
-        if (m > mlag) m = mlag;
-        p.M = (int)m;
-        p.num_super = (p.num_tiles + m - 1) / m;
+        if (M > mlag) M = mlag;
     }
-    const int64_t US = (int64_t)p.M * geo.U;  // lane length of a super-tile
-    mcol<T>(ITEMS, K, p.bc);
-    mcol<T>(geo.Uw, K, p.bw);
-    mcol<T>(geo.U, K, p.bu);
-    mcol<T>(US, K, p.bus);
-    constexpr int V = LB<T, K>::V;
-    {   // window rows: enough for the carry warps together to cover the P-1 aggregates in one round trip
-        const uint64_t P = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
-        const uint64_t rows = (P + geo.Wn - 1) / geo.Wn;
-        uint64_t vr = (rows + NCARRY - 1) / NCARRY;
-        if (vr < 1) vr = 1;
-        if (vr > (uint64_t)V) vr = V;
-        vr = V;  // measured: the full register budget per round trip beats spreading rows over warps
-        if (const char* env = getenv("SAM_VR")) { const int f = atoi(env); if (f >= 1 && f <= V) vr = f; }
-        p.Vr = (int)vr;
-    }
-    for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * p.Vr * US, K, p.bwinj[j]);
-    mcol<T>((int64_t)(grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super) - 1) * US, K, p.bprev);
-    mcol<T>((int64_t)geo.Wn * US, K, p.bwn);
-    for (int v = 0; v < 32; ++v) {
-        T b[K];
-        mcol<T>((int64_t)v * ITEMS, K, b);
-        for (int d = 0; d < K; ++d) p.bt[d][v] = b[d];
-    }
-    for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, p.bq[q]);
-    for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, p.bl[j]);
-    for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, p.bsub[j]);
-    for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * ITEMS, K, p.bks[l]);
-    for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, p.bkw[l]);
-
-    // persistent: one CTA per SM (warp-specialised: geo.W compute warps + producer, aggregator, carry warps)
-    // carry warps cooperate on each super-tile when its fold spans 3 or more windows
-    {
-        const uint64_t wv = (uint64_t)geo.Wn * V;
-        const uint64_t P = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
-        p.coop = 1;  // measured faster for every config tried, also single-window folds
-        (void)P; (void)wv;
-        if (const char* env = getenv("SAM_COOP")) p.coop = atoi(env) != 0;  // experiments
-    }
+    const uint64_t num_super = (num_tiles + M - 1) / M;
+    // measured: the full register budget per round trip beats spreading window rows over warps
+    int Vr = V;
+    if (kn.vr >= 1 && kn.vr <= V) Vr = kn.vr;
     // Static schedule (CTA b owns super-tiles b, b+P, ...): every CTA waits on aggregates of the
-    // others, so all P CTAs must be co-resident -- a cooperative launch guarantees it (or fails).
-    const uint64_t grid = grid_of(info.max_blocks_per_sm, a.num_sms, p.num_super);
-    cudaLaunchConfig_t cfg;
-    memset(&cfg, 0, sizeof(cfg));
-    cfg.gridDim = dim3((unsigned)grid);
-    cfg.blockDim = dim3((Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32);
-    cfg.dynamicSmemBytes = S::BYTES;
-    cfg.stream = a.stream;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeCooperative;
-    attr[0].val.cooperative = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, sam_scan_kernel<T, K, VEC>, p);
-    if (launches && e == cudaSuccess) ++*launches;
-    return e != cudaSuccess ? e : cudaGetLastError();
+    // others, so all P CTAs must be co-resident -- a cooperative launch guarantees it or fails; on
+    // failure the grid shrinks (the schedule is correct for any P) and the cap is remembered.
+    uint64_t P = grid_of(maxb, a.num_sms, num_super);
+    for (;;) {
+        {
+            uint64_t cap = grid_cap(dev);
+            const uint64_t dcap = debug_grid_limit() ? debug_grid_cap(dev) : 0;
+            if (dcap && (!cap || dcap < cap)) cap = dcap;
+            if (cap && P > cap) P = cap;
+        }
+        Params<T, K> p;
+        {
+            std::lock_guard<std::mutex> lk(info.mu);
+            const ShapeKey key{dev, a.s, (int)M, Vr, P};
+            auto it = tables.find(key);
+            if (it == tables.end()) {
+                Params<T, K>* t = new Params<T, K>;
+                memset(t, 0, sizeof(*t));
+                t->s = geo.s; t->G = geo.G; t->logG = geo.logG; t->sp = geo.sp; t->c = geo.c; t->logc = geo.logc;
+                t->Pw = geo.Pw; t->W = geo.W; t->Wn = geo.Wn; t->U = geo.U; t->T_ = geo.T; t->Uw = geo.Uw;
+                t->M = (int)M;
+                t->Vr = Vr;
+                t->coop = kn.coop >= 0 ? kn.coop : 1;  // measured faster for every config tried
+                const int64_t US = (int64_t)M * geo.U;  // lane length of a super-tile
+                mcol<T>(ITEMS, K, t->bc);
+                mcol<T>(geo.Uw, K, t->bw);
+                mcol<T>(geo.U, K, t->bu);
+                mcol<T>(US, K, t->bus);
+                for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * Vr * US, K, t->bwinj[j]);
+                mcol<T>((int64_t)(P - 1) * US, K, t->bprev);
+                mcol<T>((int64_t)geo.Wn * US, K, t->bwn);
+                for (int v = 0; v < 32; ++v) {
+                    T b[K];
+                    mcol<T>((int64_t)v * ITEMS, K, b);
+                    for (int d = 0; d < K; ++d) t->bt[d][v] = b[d];
+                }
+                for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, t->bq[q]);
+                for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, t->bl[j]);
+                for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, t->bsub[j]);
+                for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * ITEMS, K, t->bks[l]);
+                for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, t->bkw[l]);
+                it = tables.emplace(key, t).first;
+            }
+            memcpy(&p, it->second, sizeof(p));
+        }
+        // per-call fields
+        p.in = (const T*)a.in;
+        p.out = (T*)a.out;
+        p.n = a.n;
+        p.h = h;
+        p.num_tiles = num_tiles;
+        p.num_super = num_super;
+        p.delta = (uint32_t)(((uintptr_t)a.in - h * sizeof(T)) & 15);
+        p.inclusive = a.inclusive;
+        p.store_mode = a.store_mode;
+        p.claim_slack = kn.claim_slack;
+        p.seed = (const T*)a.seed;
+        p.final_state = (T*)a.final_state;
+        for (int m = 0; m < MAXS; ++m) {
+            p.last_e[m] = -1;
+            if (m < a.s && a.n > 0) {
+                const int64_t eend = (int64_t)(h + a.n - 1);
+                const int64_t le = eend - ((eend - m) % a.s + a.s) % a.s;
+                if (le >= (int64_t)h && le >= 0) p.last_e[m] = le;
+            }
+        }
+        p.carry = a.carry;
+        p.carry_words = a.carry_words;
+        p.tile_ctr = a.tile_ctr;
+        p.done_ctr = a.done_ctr;
+        p.epoch_ptr = a.epoch_ptr;
+        p.reset_ctr = a.reset_ctr;
+        p.trace = a.trace;
+        p.stress = debug_stress();
+
+        cudaLaunchConfig_t cfg;
+        memset(&cfg, 0, sizeof(cfg));
+        cfg.gridDim = dim3((unsigned)P);
+        cfg.blockDim = dim3((Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32);
+        cfg.dynamicSmemBytes = S::BYTES;
+        cfg.stream = a.stream;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        const bool simulated = debug_grid_limit() && P > debug_grid_limit();
+        cudaError_t e = simulated ? cudaErrorCooperativeLaunchTooLarge : cudaLaunchKernelEx(&cfg, sam_scan_kernel<T, K, VEC>, p);
+        if (e == cudaErrorCooperativeLaunchTooLarge && P > 1) {
+            if (!simulated) cudaGetLastError();  // clear, retry with a smaller co-resident grid
+            P = P - (P + 3) / 4;
+            (simulated ? debug_grid_cap(dev) : grid_cap(dev)) = P;
+            continue;
+        }
+        if (launches && e == cudaSuccess) ++*launches;
+        return e != cudaSuccess ? e : cudaGetLastError();
+    }
 }
 
 // tuple 1 with a 16-B aligned input: the 128-bit shared-memory variant
 template <typename T, int K>
 cudaError_t launch_scan_tk(const LaunchArgs& a, uint64_t* launches) {
-    const bool vec = a.s == 1 && ((uintptr_t)a.in & 15) == 0 && getenv("SAM_NO_VEC") == nullptr;
+    const bool vec = a.s == 1 && ((uintptr_t)a.in & 15) == 0 && !knobs().no_vec;
     return vec ? launch_scan_impl<T, K, true>(a, launches) : launch_scan_impl<T, K, false>(a, launches);
 }
 

@@ -43,41 +43,56 @@ def shard_offsets(n_local: int, group=None, device=None) -> tuple[int, int]:
     return int(sum(lens[:rank])), int(sum(lens))
 
 
+def _gather(t: torch.Tensor, group=None) -> torch.Tensor:
+    """all_gather_into_tensor in rank order.  NCCL moves CUDA tensors over NVLink; a gloo group
+    (CPU tests, or several ranks sharing one GPU) gets the bytes staged through host memory."""
+    world = dist.get_world_size(group)
+    if t.is_cuda and dist.get_backend(group) == "gloo":
+        h = t.cpu()
+        out = torch.empty(world * h.numel(), dtype=h.dtype)
+        dist.all_gather_into_tensor(out, h, group=group)
+        return out.to(t.device, non_blocking=False)
+    out = torch.empty(world * t.numel(), dtype=t.dtype, device=t.device)
+    dist.all_gather_into_tensor(out, t, group=group)
+    return out
+
+
 def exchange_payloads(payload: torch.Tensor, group=None) -> torch.Tensor:
     """All-gather the per-rank payloads (uint8) in rank order (NCCL over NVLink on GPUs)."""
-    world = dist.get_world_size(group)
-    gathered = torch.empty(world * payload.numel(), dtype=torch.uint8, device=payload.device)
-    dist.all_gather_into_tensor(gathered, payload, group=group)
-    return gathered
+    return _gather(payload, group)
 
 
 def scan_sharded(x_local: torch.Tensor, order: int = 1, tuple: int = 1, inclusive: bool = True,
                  group=None, global_offset: int | None = None, out: torch.Tensor | None = None,
                  stream=None) -> torch.Tensor:
-    """Scan of the global array whose contiguous shard `x_local` this rank holds."""
+    """Scan of the global array whose contiguous shard `x_local` this rank holds.  Every step --
+    state pass, all-gather, seeded scan -- is issued on `stream` (default: the current stream), so
+    the collective is ordered after the payload it sends and before the scan that reads it."""
     if not x_local.is_cuda or x_local.dim() != 1 or not x_local.is_contiguous():
         raise SamError(-1, "x_local must be a 1-D contiguous CUDA tensor")
-    world = dist.get_world_size(group)
-    rank = dist.get_rank(group)
-    if global_offset is None:
-        global_offset, _ = shard_offsets(x_local.numel(), group, device=x_local.device)
-    if out is None:
-        out = torch.empty_like(x_local)
-    dc = dtype_code(x_local.dtype)
-    st = _stream_ptr(stream)
-    n = x_local.numel()
-    if world == 1:
+    st_obj = stream if stream is not None else torch.cuda.current_stream(x_local.device)
+    with torch.cuda.stream(st_obj):
+        world = dist.get_world_size(group)
+        rank = dist.get_rank(group)
+        if global_offset is None:
+            global_offset, _ = shard_offsets(x_local.numel(), group, device=x_local.device)
+        if out is None:
+            out = torch.empty_like(x_local)
+        dc = dtype_code(x_local.dtype)
+        st = _stream_ptr(st_obj)
+        n = x_local.numel()
+        if world == 1:
+            sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x_local.data_ptr()),
+                           ctypes.c_void_p(out.data_ptr()), n, global_offset, None, 0, 1, st)
+            return out
+        pb = sam_shard_payload_bytes(dc, order, tuple)
+        payload = torch.empty(pb, dtype=torch.uint8, device=x_local.device)
+        sam_shard_state(dc, order, tuple, ctypes.c_void_p(x_local.data_ptr()), n, global_offset,
+                        ctypes.c_void_p(payload.data_ptr()), st)
+        gathered = exchange_payloads(payload, group)
         sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x_local.data_ptr()),
-                       ctypes.c_void_p(out.data_ptr()), n, global_offset, None, 0, 1, st)
-        return out
-    pb = sam_shard_payload_bytes(dc, order, tuple)
-    payload = torch.empty(pb, dtype=torch.uint8, device=x_local.device)
-    sam_shard_state(dc, order, tuple, ctypes.c_void_p(x_local.data_ptr()), n, global_offset,
-                    ctypes.c_void_p(payload.data_ptr()), st)
-    gathered = exchange_payloads(payload, group)
-    sam_shard_scan(dc, order, tuple, inclusive, ctypes.c_void_p(x_local.data_ptr()),
-                   ctypes.c_void_p(out.data_ptr()), n, global_offset, ctypes.c_void_p(gathered.data_ptr()),
-                   rank, world, st)
+                       ctypes.c_void_p(out.data_ptr()), n, global_offset, ctypes.c_void_p(gathered.data_ptr()),
+                       rank, world, st)
     return out
 
 
@@ -115,34 +130,48 @@ def shard_tail(x_local: torch.Tensor) -> torch.Tensor:
     return t
 
 
-def halo_from_tails(tails: torch.Tensor, lens: list[int], rank: int, ks: int) -> torch.Tensor:
+def halo_from_tails(tails: torch.Tensor, lens, rank: int, ks: int) -> torch.Tensor:
     """Halo of `rank` (the ks elements preceding its shard, zero-left-padded) from the gathered
-    tails [world, TAIL] and shard lengths: the suffix of the valid tails of ranks < rank.  The
-    valid tail of a shard is all of it when n < TAIL, so the concatenation ends with the last
-    TAIL elements of the global prefix."""
-    parts = [tails[r, TAIL - min(lens[r], TAIL):] for r in range(rank)]
-    z = torch.zeros(ks, dtype=tails.dtype, device=tails.device)
-    cat = torch.cat([z] + parts)
-    return cat[cat.numel() - ks:].contiguous()
+    tails [world, TAIL] and shard lengths (a list, or an int64 tensor on the tails' device): the
+    suffix of the valid tails of ranks < rank.  The valid tail of a shard is all of it when
+    n < TAIL, so the concatenation ends with the last TAIL elements of the global prefix.  Pure
+    tensor indexing, no host synchronisation."""
+    if rank == 0:
+        return torch.zeros(ks, dtype=tails.dtype, device=tails.device)
+    lens_t = torch.as_tensor(lens, dtype=torch.int64, device=tails.device)[:rank]
+    pos = torch.arange(TAIL, device=tails.device)
+    valid = pos[None, :] >= (TAIL - torch.clamp(lens_t, max=TAIL))[:, None]  # [rank, TAIL]
+    flat = tails[:rank].reshape(-1)
+    v = valid.reshape(-1)
+    # rc[i] = number of valid elements at or after i; the halo takes those with rc <= ks
+    rc = torch.flip(torch.cumsum(torch.flip(v.to(torch.int64), [0]), 0), [0])
+    take = v & (rc <= ks)
+    dest = torch.where(take, ks - rc, torch.full_like(rc, ks))  # slot ks = discard
+    halo = torch.zeros(ks + 1, dtype=tails.dtype, device=tails.device)
+    halo.scatter_(0, dest, torch.where(take, flat, torch.zeros_like(flat)))
+    return halo[:ks].contiguous()
 
 
 def delta_encode_sharded(x_local: torch.Tensor, order: int = 1, tuple: int = 1, group=None,
                          out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """Delta encoding (k-th order, stride s) of the global array whose contiguous shard `x_local`
-    this rank holds: one all-gather of shard tails and lengths, then sam_delta_encode_halo."""
+    this rank holds: ONE all-gather of [n_r | shard tail] records, the halo assembled on the device
+    (no host synchronisation), then sam_delta_encode_halo -- all on `stream`."""
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
     if world == 1:
         return delta_encode(x_local, order, tuple, out=out, stream=stream)
-    tail = shard_tail(x_local)
-    tails = torch.empty(world * TAIL, dtype=x_local.dtype, device=x_local.device)
-    dist.all_gather_into_tensor(tails, tail, group=group)
-    tails = tails.view(world, TAIL)
-    n = torch.tensor([x_local.numel()], dtype=torch.int64, device=x_local.device)
-    lens_t = torch.empty(world, dtype=torch.int64, device=x_local.device)
-    dist.all_gather_into_tensor(lens_t, n, group=group)
-    halo = halo_from_tails(tails, lens_t.tolist(), rank, order * tuple)
-    return delta_encode(x_local, order, tuple, out=out, stream=stream, halo=halo)
+    st_obj = stream if stream is not None else torch.cuda.current_stream(x_local.device)
+    with torch.cuda.stream(st_obj):
+        w = x_local.element_size()
+        rec = torch.empty(8 + TAIL * w, dtype=torch.uint8, device=x_local.device)
+        rec[:8].view(torch.int64).fill_(x_local.numel())
+        rec[8:].view(x_local.dtype).copy_(shard_tail(x_local))
+        recs = _gather(rec, group).view(world, 8 + TAIL * w)
+        lens_t = recs[:, :8].contiguous().view(torch.int64).reshape(world)
+        tails = recs[:, 8:].contiguous().view(x_local.dtype).reshape(world, TAIL)
+        halo = halo_from_tails(tails, lens_t, rank, order * tuple)
+        return delta_encode(x_local, order, tuple, out=out, stream=st_obj, halo=halo)
 
 
 def delta_virtual_shards(x: torch.Tensor, bounds: list[int], order: int = 1, tuple: int = 1) -> torch.Tensor:

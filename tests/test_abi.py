@@ -146,3 +146,23 @@ def test_host_fold_floats_close():
         _, run = oracle.scan(x[: bounds[rank]], k, s, True, phase=0)
         ref = run.reshape(k, s).T.astype(np.float64)
         assert np.allclose(seed.reshape(s, k), ref, rtol=1e-12, atol=0)
+
+
+def test_workspace_size_and_ws_validation():
+    """sam_scan_workspace_size / sam_scan_ws: sizes grow with n and with k*s, and
+    sam_scan_ws validates its workspace synchronously, before any CUDA call."""
+    S = _lib()
+    L = S.lib()
+    sz = [S.sam_scan_workspace_size(S.SAM_I64, 4, 4, n) for n in (1, 1 << 20, 1 << 30, 1 << 33)]
+    assert sz == sorted(sz) and sz[0] >= 1024
+    assert S.sam_scan_workspace_size(S.SAM_I32, 8, 8, 1 << 20) >= S.sam_scan_workspace_size(S.SAM_I32, 1, 1, 1 << 20)
+    with pytest.raises(S.SamError):
+        S.sam_scan_workspace_size(S.SAM_I32, 9, 1, 10)
+    buf = (ctypes.c_int64 * 512)()
+    base = ctypes.addressof(buf)
+    need = S.sam_scan_workspace_size(S.SAM_I32, 1, 1, 16)
+    assert L.sam_scan_ws(0, 1, 1, 1, base, base + 2048, 16, None, need, None) == -1        # null ws
+    assert L.sam_scan_ws(0, 1, 1, 1, base, base + 2048, 16, base + 8, need, None) == -1    # misaligned ws
+    assert L.sam_scan_ws(0, 1, 1, 1, base, base + 2048, 16, base + 16, need - 8, None) == -1  # too small
+    assert "workspace" in S.sam_last_error()
+    assert L.sam_scan_ws(0, 1, 1, 1, base, base, 0, None, 0, None) == 0                   # n == 0: no-op

@@ -96,3 +96,27 @@ def test_C5_sharded_order4_tuple4():
             assert np.array_equal(ys.cpu().numpy().view(ref.dtype), ref)
         del x, ys, y1
         torch.cuda.empty_cache()
+
+
+def test_C5_2p33_int64_order4_tuple4_single_gpu():
+    """n = 2^33 > 2^32 elements (C5 strong at p = 1): 64 GiB in + 64 GiB
+    out in HBM, one launch.  Verified against the chunked oracle (the same serial loop with its
+    per-(pass, lane) running sums carried across chunks) on D2H chunks of the output."""
+    import paper_conf_pldi_malekiyb16_b200 as S
+
+    free, _ = torch.cuda.mem_get_info()
+    n = 1 << 33
+    if free < 2 * 8 * n + (4 << 30):
+        pytest.skip(f"needs ~132 GiB free HBM, have {free / 2**30:.0f} GiB")
+    k, s = 4, 4
+    x = synth.make_torch(n, "i64", "uniform", seed=synth.SEED_BASE + 9, device="cuda")
+    y = torch.empty_like(x)
+    S.scan(x, k, s, True, out=y)
+    torch.cuda.synchronize()
+    run = None
+    chunk = 1 << 28
+    for off in range(0, n, chunk):
+        xc = x[off:off + chunk].cpu().numpy()
+        ref, run = oracle.scan(xc, k, s, True, phase=off % s, run=run)
+        got = y[off:off + chunk].cpu().numpy().view(ref.dtype)
+        assert np.array_equal(got, ref), f"mismatch in chunk at {off}"

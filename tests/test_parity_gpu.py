@@ -14,12 +14,13 @@ import pytest
 
 torch = pytest.importorskip("torch")
 
+import oracle
 import synth
 from tests.helpers import DT, compare, torch_dtype
 
 pytestmark = pytest.mark.gpu
 
-N_SWEEP = 20011  # prime: ragged for every s, >= 5 tiles for every s
+N_SWEEP = 40009  # prime: ragged for every s; >= 5 tiles for every s (largest tile: 7168 elements)
 
 
 def sam():
@@ -200,14 +201,143 @@ def test_scan_host_pipeline(name):
         compare(name, xn, y.numpy(), k, s, True)
 
 
-@pytest.mark.parametrize("name,k,s", [("i32", 1, 1), ("i32", 2, 1), ("i32", 3, 1), ("i64", 1, 1), ("i64", 4, 1),
-                                      ("i64", 1, 3), ("i64", 2, 8), ("i32", 8, 1), ("i64", 8, 5)])
+N_MULTI = 148 * 3 * 7168 * 3 + 4099  # > 3 super-tiles per CTA on 148 SMs for every (dtype, s)
+
+
+def _multi_round_input(name, k, s):
+    """Inputs for the multi-round parity grid.  Ints: full-range bits (wraparound).  Floats: signed
+    values in [-1, 1) scaled by a power of two so the order-k partial sums stay finite (R9)."""
+    if name in ("i32", "i64"):
+        return synth.make(N_MULTI, name, "uniform", seed=synth.SEED_BASE + 4242 + 16 * k + s)
+    x = synth.make(N_MULTI, name, "unif01", seed=synth.SEED_BASE + 4343 + 16 * k + s)
+    x = (x * DT[name](2) - DT[name](1))
+    # order-k growth ~ (n/s)^k / k!: keep max |y| far below the format's range
+    scale = {"f32": 2.0 ** -(6 * k), "f64": 2.0 ** -(6 * k)}[name]
+    return (x * DT[name](scale)).astype(DT[name])
+
+
+@pytest.mark.parametrize("name", ["i32", "i64", "f32", "f64"])
+@pytest.mark.parametrize("k", range(1, 9))
+@pytest.mark.parametrize("s", [1, 3, 4, 8])
 def test_multi_round_schedule(name, k, s):
-    # > 3 super-tiles per CTA on 148 SMs (tiles of 3328..7168 elements, super-tiles of 2-3 tiles)
-    n = 148 * 3 * 7168 * 3 + 4099
-    x = synth.make(n, name, "uniform", seed=synth.SEED_BASE + 4242 + 16 * k + s)
+    """The full carry schedule (hand-off of a CTA's own inclusive state across >= 3 rounds, multi-
+    window folds of the P-1 aggregates in between) for every dtype x order x tuple class, inclusive
+    and exclusive, element by element against the oracle."""
+    x = _multi_round_input(name, k, s)
     for inclusive in (True, False):
         compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
+
+
+@pytest.mark.parametrize("name", ["f32", "f64"])
+@pytest.mark.parametrize("k", [1, 2])
+@pytest.mark.parametrize("s", [1, 3, 4, 8])
+def test_multi_round_float_exact(name, k, s):
+    """Integer-valued +-1 inputs at the multi-round size: bit-exact wherever every partial sum of
+    every association order is an integer below 2^24 / 2^53 (SURVEY §8(c) floats): order 1 via the
+    per-lane prefix range, order 2 via the order-2 scan of |x|."""
+    x = synth.make(N_MULTI, name, "pm1int", seed=synth.SEED_BASE + 4444 + 16 * k + s)
+    lim = 2.0 ** (24 if name == "f32" else 53)
+    if k == 1:
+        ref = oracle.scan(x, 1, s, True)[0].astype(np.float64)
+        exact = all((np.ptp(np.concatenate([[0.0], ref[m::s]])) < lim) for m in range(s))
+    else:
+        exact = float(oracle.scan(np.abs(x), k, s, True)[0].max()) < lim
+    for inclusive in (True, False):
+        compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive, exact_float=exact)
+
+
+@pytest.mark.parametrize("grid", [1, 2, 7, 37, 100])
+@pytest.mark.parametrize("name,k,s", [("i32", 1, 1), ("i64", 4, 4), ("i32", 8, 3), ("f64", 2, 8)])
+def test_reduced_grid_fallback(grid, name, k, s):
+    """The cooperative-launch fallback (not all SMs available): grids above `grid` are
+    refused, the launch shrinks the grid and retries; SAM's schedule must be exact for any P."""
+    S = sam()
+    x = synth.make(1 << 21, name, "uniform" if name[0] == "i" else "small", seed=synth.SEED_BASE + grid + k)
+    S.sam_debug_limit_grid(grid)
+    try:
+        for inclusive in (True, False):
+            compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
+    finally:
+        S.sam_debug_limit_grid(0)
+
+
+@pytest.mark.parametrize("name,k,s", [("i32", 1, 1), ("i64", 1, 1), ("i32", 4, 1), ("i64", 8, 1), ("i64", 4, 4),
+                                      ("i32", 2, 3), ("i64", 1, 5), ("f64", 3, 8)])
+def test_stress_random_delays(name, k, s):
+    """Randomised delays at every pipeline hand-over (sam_debug_set_stress), 100 seeds: every run
+    equals the oracle-checked result bit for bit (SURVEY §4 tier 5)."""
+    S = sam()
+    xn = synth.make(148 * 2 * 7168 + 999, name, "uniform" if name[0] == "i" else "small", seed=synth.SEED_BASE + 17)
+    x = torch.from_numpy(xn).cuda()
+    ref = S.scan(x, k, s, True)
+    torch.cuda.synchronize()
+    compare(name, xn, ref.cpu().numpy(), k, s, True)
+    try:
+        for seed in range(1, 101):
+            S.sam_debug_set_stress(seed)
+            y = S.scan(x, k, s, True)
+            torch.cuda.synchronize()
+            assert torch.equal(y.view(torch.uint8), ref.view(torch.uint8)), f"stress seed {seed} differs"
+    finally:
+        S.sam_debug_set_stress(0)
+
+
+def test_explicit_workspace_and_graph_growth():
+    """sam_scan_ws: caller-owned workspace (zero-filled once), no allocation or synchronisation in
+    the call, so a graph can be captured for a LARGER n than any earlier call (the cached workspace
+    would need a grow + sync there)."""
+    S = sam()
+    dc = S.SAM_I32
+    nmax = 3_000_017
+    wsb = S.sam_scan_workspace_size(dc, 3, 2, nmax)
+    ws = torch.zeros(wsb, dtype=torch.uint8, device="cuda")
+    for n in (1000, 77777, nmax):
+        xn = synth.make(n, "i32", "uniform", seed=n)
+        x = torch.from_numpy(xn).cuda()
+        y = torch.empty_like(x)
+        S.sam_scan_ws(dc, 3, 2, True, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(y.data_ptr()), n,
+                      ctypes.c_void_p(ws.data_ptr()), wsb, S._stream_ptr())
+        torch.cuda.synchronize()
+        compare("i32", xn, y.cpu().numpy(), 3, 2, True)
+    # capture on a fresh stream with the explicit workspace, never used on that stream before
+    xn = synth.make(nmax, "i32", "uniform", seed=4)
+    x = torch.from_numpy(xn).cuda()
+    y = torch.empty_like(x)
+    st = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=st):
+        S.sam_scan_ws(dc, 3, 2, False, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(y.data_ptr()), nmax,
+                      ctypes.c_void_p(ws.data_ptr()), wsb, S._stream_ptr(st))
+    for _ in range(5):
+        y.zero_()
+        g.replay()
+    torch.cuda.synchronize()
+    compare("i32", xn, y.cpu().numpy(), 3, 2, False)
+
+
+def test_epoch_wraparound_resets_carry_words():
+    """the 32-bit launch epoch wraps after 2^32 launches of a workspace.  Put the epoch
+    just before the wrap and fill the carry words with words tagged 1..3 (what launches 2^32 ago
+    would have left): the wrap launch zeroes the words first, so no stale word validates."""
+    S = sam()
+    dc = S.SAM_I64
+    n = 1 << 21
+    wsb = S.sam_scan_workspace_size(dc, 2, 3, n)
+    ws = torch.zeros(wsb // 8, dtype=torch.int64, device="cuda")
+    carry = ws[1024 // 8:]
+    stale = torch.randint(0, 1 << 31, (carry.numel(),), dtype=torch.int64, device="cuda")
+    carry.copy_(stale | (torch.randint(1, 4, (carry.numel(),), dtype=torch.int64, device="cuda") << 32))
+    hdr32 = ws[:4].view(torch.int32)
+    hdr32[3] = -3  # epoch word (offset 12) = 0xFFFFFFFD
+    xn = synth.make(n, "i64", "uniform", seed=123)
+    x = torch.from_numpy(xn).cuda()
+    for it in range(6):  # tags FE, FF, then the wrap launch (reset, tag 1), 2, 3, 4
+        y = torch.empty_like(x)
+        S.sam_scan_ws(dc, 2, 3, True, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(y.data_ptr()), n,
+                      ctypes.c_void_p(ws.data_ptr()), wsb, S._stream_ptr())
+        torch.cuda.synchronize()
+        compare("i64", xn, y.cpu().numpy(), 2, 3, True)
+    assert int(hdr32[3].item()) == 4
 
 
 @pytest.mark.parametrize("name,k,s", [("f32", 1, 1), ("f64", 1, 1), ("f32", 2, 3), ("f64", 4, 4)])
