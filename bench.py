@@ -122,6 +122,80 @@ class ClockSampler:
                 "power_w": statistics.median(lw) if lw else None}
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+
+    return platform.processor() or platform.machine()
+
+
+# Every BASELINE.json config, one line each in the `sweep` key: name, dtype,
+# log2 n, order, tuple.  C3: int32/int64 orders 1..8; C4: int64 tuples 1..8 at orders 1, 2 and
+# fp32/fp64 tuples at order 1; C5: int64 order 4 tuple 4 at 2^30 (one GPU's weak-scaling share) and
+# at 2^33 (the strong-scaling total, > 2^32 elements, 128 GiB of HBM).
+SWEEP = ([(f"C3 i32 k={k}", "i32", 28, k, 1) for k in range(1, 9)] +
+         [(f"C3 i64 k={k}", "i64", 28, k, 1) for k in range(1, 9)] +
+         [(f"C4 i64 k={k} s={s}", "i64", 28, k, s) for k in (1, 2) for s in range(1, 9)] +
+         [(f"C4 {d} k=1 s={s}", d, 28, 1, s) for d in ("f32", "f64") for s in range(1, 9)] +
+         [("C5 i64 k=4 s=4 n=2^30", "i64", 30, 4, 4), ("C5 i64 k=4 s=4 n=2^33", "i64", 33, 4, 4)])
+
+
+def run_sweep(sam, synth, torch, peak, reps=5):
+    """Kernel-only throughput of every config (CUDA events on the launching stream, inputs in HBM,
+    > L2), against a memcpy of the same bytes and the measured copy peak."""
+    import ctypes
+
+    out = []
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    memcpy_cache = {}
+    for name, dt, logn, k, s in SWEEP:
+        n = 1 << logn
+        w = W_BYTES[dt]
+        free, _ = torch.cuda.mem_get_info()
+        if free < 2 * n * w + (2 << 30):
+            out.append({"config": name, "skipped": f"needs {2 * n * w / 2**30:.0f} GiB free HBM"})
+            continue
+        x = synth.make_torch(n, dt, "uniform" if dt[0] == "i" else "unif01", seed=synth.SEED_BASE + 2, device="cuda")
+        y = torch.empty_like(x)
+        st = torch.cuda.current_stream()
+        sp = ctypes.c_void_p(st.cuda_stream)
+        dc = sam.dtype_code(x.dtype)
+        P = lambda t: ctypes.c_void_p(t.data_ptr())
+        for _ in range(2):
+            sam.sam_scan(dc, k, s, True, P(x), P(y), n, sp)
+        torch.cuda.synchronize()
+        e0.record(st)
+        for _ in range(reps):
+            sam.sam_scan(dc, k, s, True, P(x), P(y), n, sp)
+        e1.record(st)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / reps
+        key = (n, w)
+        if key not in memcpy_cache:
+            for _ in range(2):
+                y.copy_(x)
+            e0.record(st)
+            for _ in range(reps):
+                y.copy_(x)
+            e1.record(st)
+            torch.cuda.synchronize()
+            memcpy_cache[key] = e0.elapsed_time(e1) / reps
+        gbs = 2 * w * n / (ms * 1e-3) / 1e9
+        out.append({"config": name, "n": n, "order": k, "tuple": s, "dtype": DTYPE_NAME[dt],
+                    "gvalues_s": n / (ms * 1e-3) / 1e9, "gbs": gbs, "ms": ms,
+                    "frac_of_memcpy": memcpy_cache[key] / ms, "roofline_frac": gbs / peak,
+                    "traffic": ncu_traffic(name)})
+        del x, y
+        torch.cuda.empty_cache()
+    return out
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -176,6 +250,7 @@ def main():
     ap.add_argument("--config", default="C2", choices=sorted(CONFIGS))
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the per-config sweep (C3/C4/C5) key")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -381,9 +456,27 @@ def main():
             orun(xs)
             ts.append(time.perf_counter() - t0)
         cpu = {"value": sample / statistics.median(ts) / 1e9, "unit": "Gvalues/s", "cores": 1, "kind": "oracle",
-               "sample": f"first 2^27 elements of the same input, serial oracle (oracle/sam_oracle.c), median of 3"}
+               "sample": f"first 2^27 elements of the same input, serial oracle (oracle/sam_oracle.c), median of 3",
+               "cpu_model": cpu_model(), "nproc": os.cpu_count()}
+        if dt in ("i32", "i64") and not delta and incl:
+            # context only: all host cores, k passes of two-phase order-1 scans (oracle/cpu_allcores.c)
+            nt = os.cpu_count() or 1
+            oracle.scan_allcores(xs[: 1 << 20], k, s, threads=nt)
+            ta = []
+            for _ in range(3):
+                t0 = time.perf_counter()
+                oracle.scan_allcores(xs, k, s, threads=nt)
+                ta.append(time.perf_counter() - t0)
+            cpu["allcores"] = {"value": sample / statistics.median(ta) / 1e9, "unit": "Gvalues/s", "threads": nt,
+                               "kind": "all-cores context scan (k passes of two-phase order-1 scans, OpenMP)",
+                               "sample": "same 2^27-element sample, median of 3"}
 
     peak, peak_src = measured_peaks()
+    sweep = None
+    if world == 1 and not args.no_sweep and not delta:
+        del y
+        torch.cuda.empty_cache()
+        sweep = run_sweep(sam, synth, torch, peak)
     alg_bytes = 2 * w * n_local
     achieved = alg_bytes / (kavg * 1e-3) / 1e9
     if rank == 0:
@@ -404,6 +497,7 @@ def main():
                          "kernel": "sam::delta_kernel" if delta else "sam::sam_scan_kernel", "kernel_ms": kavg,
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
             "cpu_baseline": cpu,
+            "sweep": sweep,
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk.summary(),

@@ -26,6 +26,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "sam_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
+_SRC_MT = os.path.join(_HERE, "cpu_allcores.c")
+_LIB_MT = os.path.join(_HERE, "liboracle_mt.so")
+_lib_mt = None
 
 
 def build(force: bool = False) -> str:
@@ -36,6 +39,39 @@ def build(force: bool = False) -> str:
                                "-fno-fast-math", "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
     return _LIB
+
+
+def build_allcores(force: bool = False) -> str:
+    """Compile the all-cores CPU context scan (OpenMP; cpu_allcores.c)."""
+    if force or not os.path.exists(_LIB_MT) or os.path.getmtime(_LIB_MT) < os.path.getmtime(_SRC_MT):
+        tmp = _LIB_MT + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O3", "-std=c11", "-fPIC", "-shared", "-fopenmp", "-o", tmp, _SRC_MT])
+        os.replace(tmp, _LIB_MT)
+    return _LIB_MT
+
+
+def scan_allcores(x: np.ndarray, k: int, s: int = 1, phase: int = 0, threads: int | None = None) -> np.ndarray:
+    """All-cores CPU context scan (inclusive, integers only): k passes of two-phase order-1 scans
+    over `threads` chunks (default: os.cpu_count()).  Returns uint32/uint64 like scan()."""
+    global _lib_mt
+    if _lib_mt is None:
+        L = ctypes.CDLL(build_allcores())
+        for name in ("allcores_scan_u32", "allcores_scan_u64"):
+            fn = getattr(L, name)
+            fn.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int]
+            fn.restype = ctypes.c_int
+        _lib_mt = L
+    x = np.ascontiguousarray(x)
+    if x.dtype.kind not in "iu":
+        raise ValueError("scan_allcores: integer data only")
+    acc = np.uint32 if x.dtype.itemsize == 4 else np.uint64
+    a = x.view(acc).copy()
+    nt = int(threads or os.cpu_count() or 1)
+    fn = _lib_mt.allcores_scan_u32 if acc is np.uint32 else _lib_mt.allcores_scan_u64
+    rc = fn(a.ctypes.data, a.size, int(k), int(s), int(phase), nt)
+    if rc != 0:
+        raise ValueError(f"allcores scan rejected arguments (rc={rc})")
+    return a
 
 
 def _load():

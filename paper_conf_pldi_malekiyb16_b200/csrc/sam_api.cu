@@ -65,6 +65,8 @@ int validate_buffers(sam_dtype dtype, const void* in, const void* out, uint64_t 
 struct Workspace {
     unsigned long long* carry = nullptr;  // tagged carry words of every tile
     size_t carry_cap = 0;                 // bytes
+    unsigned char* pend = nullptr;        // pending-state scratch (states > 16 B)
+    size_t pend_cap = 0;
     unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32][epoch u32][pad 16][seed 512 B]
 };
 
@@ -101,8 +103,9 @@ int num_sms(int dev) {
 constexpr size_t CTR_BYTES = 32 + 8 * 8 * 8;
 constexpr size_t WS_HEADER = 1024;
 
-// workspace of (current device, stream) with room for `carry_bytes` of tagged carry words
-int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out) {
+// workspace of (current device, stream) with room for `carry_bytes` of tagged carry words and
+// `pend_bytes` of pending-state scratch
+int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out, size_t pend_bytes = 0) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
@@ -131,9 +134,29 @@ int get_ws(cudaStream_t st, size_t carry_bytes, Workspace** out, int* dev_out) {
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
         ws->carry_cap = cap;
     }
+    if (pend_bytes > ws->pend_cap) {
+        e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+        if (ws->pend) cudaFree(ws->pend);
+        ws->pend = nullptr;
+        ws->pend_cap = 0;
+        e = cudaMalloc(&ws->pend, pend_bytes);
+        if (e != cudaSuccess) return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e));
+        ws->pend_cap = pend_bytes;
+    }
     *out = ws;
     *dev_out = dev;
     return SAM_OK;
+}
+
+int num_sms_of(int dev) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    return num_sms(dev);
+}
+
+// bytes of pending-state scratch a workspace holds (multiple of 256, placed after the header)
+size_t pend_area(sam_dtype d, int k, int dev) {
+    return (sam::pend_bytes((int)elem_size(d), k, num_sms_of(dev)) + 255) / 256 * 256;
 }
 
 int items_of(sam_dtype d) {
@@ -177,15 +200,20 @@ cudaError_t dispatch_k(int k, const sam::LaunchArgs& a) {
 // an explicit workspace (sam_scan_ws), or null for the cached (device, stream) workspace.
 int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void* out, uint64_t n, uint64_t g,
              const void* seed, void* final_state, int store_mode, cudaStream_t st,
-             unsigned char* ws_hdr = nullptr, unsigned long long* ws_carry = nullptr, size_t ws_carry_cap = 0) {
+             unsigned char* ws_hdr = nullptr, unsigned long long* ws_carry = nullptr, size_t ws_carry_cap = 0,
+             void* ws_pend = nullptr) {
     int dev = 0;
     if (!ws_hdr) {
         Workspace* ws = nullptr;
-        int rc = get_ws(st, carry_bytes(dtype, k, s, tiles_for(dtype, s, n + g % (uint64_t)s)), &ws, &dev);
+        int d0 = 0;
+        cudaGetDevice(&d0);
+        int rc = get_ws(st, carry_bytes(dtype, k, s, tiles_for(dtype, s, n + g % (uint64_t)s)), &ws, &dev,
+                        sam::pend_bytes((int)elem_size(dtype), k, num_sms_of(d0)));
         if (rc != SAM_OK) return rc;
         ws_hdr = ws->ctr;
         ws_carry = ws->carry;
         ws_carry_cap = ws->carry_cap;
+        ws_pend = ws->pend;
     } else {
         cudaError_t e = cudaGetDevice(&dev);
         if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
@@ -207,6 +235,7 @@ int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void*
     a.done_ctr = (unsigned int*)(ws_hdr + 8);
     a.epoch_ptr = (unsigned int*)(ws_hdr + 12);
     a.reset_ctr = (unsigned int*)(ws_hdr + 16);
+    a.pend = ws_pend;
     a.num_sms = num_sms(dev);
     a.dev = dev;
     a.trace = g_trace;
@@ -276,7 +305,9 @@ int sam_scan_workspace_size(sam_dtype dtype, int order, int tuple, uint64_t n, s
     int rc = validate_common(dtype, order, tuple);
     if (rc) return rc;
     if (!bytes) return fail(SAM_ERR_INVALID_ARG, "null bytes pointer");
-    *bytes = WS_HEADER + carry_bytes(dtype, order, tuple, tiles_for(dtype, tuple, n));
+    int dev = 0;
+    cudaGetDevice(&dev);
+    *bytes = WS_HEADER + pend_area(dtype, order, dev) + carry_bytes(dtype, order, tuple, tiles_for(dtype, tuple, n));
     return SAM_OK;
 }
 
@@ -294,8 +325,12 @@ int sam_scan_ws(sam_dtype dtype, int order, int tuple, int inclusive, const void
     if (ws_bytes < need)
         return fail(SAM_ERR_INVALID_ARG, "workspace too small (sam_scan_workspace_size gives " + std::to_string(need) + " B)");
     unsigned char* w = (unsigned char*)ws;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const size_t pa = pend_area(dtype, order, dev);
     return run_scan(dtype, order, tuple, inclusive, in, out, n, 0, nullptr, nullptr, store_mode_for(in, out),
-                    (cudaStream_t)stream, w, (unsigned long long*)(w + WS_HEADER), ws_bytes - WS_HEADER);
+                    (cudaStream_t)stream, w, (unsigned long long*)(w + WS_HEADER + pa), ws_bytes - WS_HEADER - pa,
+                    pa ? (void*)(w + WS_HEADER) : nullptr);
 }
 
 size_t sam_shard_payload_bytes(sam_dtype dtype, int order, int tuple) {

@@ -125,6 +125,9 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #define SAM_PROD_NS 16
 #endif
 // orders >= SAM_KS_MIN_K scan thread/warp k-vector states Kogge-Stone style, lower orders order by order
+#ifndef SAM_TRANSFORM
+#define SAM_TRANSFORM 1
+#endif
 #ifndef SAM_KS_MIN_K
 #define SAM_KS_MIN_K 3
 #endif
@@ -141,11 +144,28 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_LAG32
 #define SAM_LAG32 6
 #endif
+#ifndef SAM_GPEND
+#define SAM_GPEND 1
+#endif
+#ifndef SAM_LAGG
+#define SAM_LAGG 12
+#endif
+// states of 33..64 B (int64 orders 5-8) without SAM_GPEND: pending in shared memory, LAG 4
+#ifndef SAM_SMEM64
+#define SAM_SMEM64 1
+#endif
+#ifndef SAM_LAG64
+#define SAM_LAG64 4
+#endif
 template <typename T, int K> struct Lag {
     static constexpr int SB = K * (int)sizeof(T);
     static constexpr bool BIG32 = SAM_SMEM32 && SB > 16 && SB <= 32;
-    static constexpr bool SMEM = SB <= 16 || BIG32;  // pending local states in shared memory
-    static constexpr int LAG = SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : (BIG32 ? SAM_LAG32 : 4)));
+    static constexpr bool BIG64 = SAM_SMEM64 && SB > 32;
+    // states > 16 B: pending in global memory (L2-resident scratch), so the pipeline depth is not
+    // bounded by shared memory
+    static constexpr bool GPEND = SAM_GPEND && SB > 16;
+    static constexpr bool SMEM = !GPEND && (SB <= 16 || BIG32 || BIG64);  // pending local states in shared memory
+    static constexpr int LAG = GPEND ? SAM_LAGG : (SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : (BIG32 ? SAM_LAG32 : SAM_LAG64))));
     // max tiles per super-tile (look-back unit); measured: 3 for 4-byte, 2 for 8-byte elements
     static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : 2;
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
@@ -153,7 +173,7 @@ template <typename T, int K> struct Lag {
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = SMEM && !BIG32 && K >= SAM_SPLIT_MIN_K;
+    static constexpr bool SPLIT = SB <= 16 && K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
@@ -179,8 +199,15 @@ template <typename T, int K> struct LB {
     static constexpr int V = V0 < 1 ? 1 : (V0 > 16 ? 16 : V0);
 };
 
+// Coefficient / carry-fold type: fp32 scans fold their carries in double -- the binomial weights
+// of spans of many super-tiles (C(L-1+d, d), L up to n) exceed the fp32 range at high orders, and
+// double keeps the fold's rounding below the tile-local one.  Integers: the element type (mod 2^w).
+template <typename T> struct Coef { using type = T; };
+template <> struct Coef<float> { using type = double; };
+
 template <typename T, int K>
 struct Params {
+    using CT = typename Coef<T>::type;
     const T* in;
     T* out;
     uint64_t n;          // elements in this stream
@@ -197,6 +224,8 @@ struct Params {
     const T* seed;        // [s][K] state before the stream per global lane, or null
     T* final_state;       // [s][K] or null
     int64_t last_e[MAXS]; // virtual index of lane m's last element, -1 if none
+    T* pend;              // GPEND: pending local states [grid][LAG][K][TILE_THREADS] (workspace)
+    int lag;              // pipeline depth used (1..LAG): max tiles between a local scan and its carry application
     unsigned long long* carry;  // tagged carry words: [tile][m][t][agg W | incl W]
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
@@ -208,16 +237,17 @@ struct Params {
     T bc[K];              // b_d(ITEMS)
     T bw[K];              // b_d(Uw)
     T bu[K];              // b_d(U)        (one tile)
-    T bus[K];             // b_d(M*U)      (one super-tile)
-    T bwinj[NCARRY_P1][K]; // b_d(j*Wn*V*M*U), j <= NCARRY (look-back windows further)
+    CT bus[K];            // b_d(M*U)      (one super-tile)
+    CT bwinj[NCARRY_P1][K]; // b_d(j*Wn*V*M*U), j <= NCARRY (carry-fold windows further)
     int coop;             // all carry warps fold each super-tile's windows together
     int Vr;               // window rows used per round trip (<= V)
-    T bprev[K];           // b_d((P-1)*M*U): from this CTA's previous super-tile to the one before S
-    T bwn[K];             // b_d(Wn*M*U)   (one window row further)
+    CT bprev[K];          // b_d((P-1)*M*U): from this CTA's previous super-tile to the one before S
+    CT bwn[K];            // b_d(Wn*M*U)   (one window row further)
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
+    T bn[K][32];          // b_d(-(v+1)*ITEMS), v < Pw    ([d][v]; integer similarity transform)
     T bq[8][K];           // b_d(q*Uw),     q < c
-    T bl[32][K];          // b_d(j*M*U),    j < Wn
-    T bsub[8][K];         // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
+    CT bl[32][K];         // b_d(j*M*U),    j < Wn
+    CT bsub[8][K];        // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
     T bks[5][K];          // b_d(2^l*ITEMS) (Kogge-Stone warp scan of thread states, K >= 3)
     T bkw[3][K];          // b_d(2^l*Uw)    (Kogge-Stone combine of warp states, K >= 3)
 };
@@ -326,6 +356,25 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
+// CTA-scope flags in shared memory (end-of-stream, progress counters, hand-off stamps): relaxed
+// atomic accesses (morally strong in the PTX memory model, and visible as such to racecheck), the
+// data they guard ordered by fences (writer: fence before the flag; reader: flag before the data)
+__device__ __forceinline__ int flag_ld(const volatile int* p) {
+    int v;
+    asm volatile("ld.relaxed.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32((const void*)p)) : "memory");
+    return v;
+}
+__device__ __forceinline__ int flag_ld_acq(const volatile int* p) {
+    int v;
+    asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32((const void*)p)) : "memory");
+    return v;
+}
+__device__ __forceinline__ void flag_st_rel(volatile int* p, int v) {
+    asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32((const void*)p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ void flag_st(volatile int* p, int v) {
+    asm volatile("st.relaxed.cta.shared.b32 [%0], %1;" ::"r"(smem_u32((const void*)p)), "r"(v) : "memory");
+}
 __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
     unsigned long long a;
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(a) : "l"(p) : "memory");
@@ -386,10 +435,11 @@ template <> struct IsInt<uint64_t> { static constexpr bool value = true; };
 // ------------------------------------------------------------------------------------------
 // shared-memory layout
 // ------------------------------------------------------------------------------------------
-template <typename T, int K, bool VEC, int NB2_>
+template <typename T, int K, bool VEC, int NB1_, int NB2_>
 struct SmemL {
+    using CT = typename Coef<T>::type;
     static constexpr int ITEMS = Items<T, VEC>::V;
-    static constexpr int NB1 = Lag<T, K>::NB1;
+    static constexpr int NB1 = NB1_;
     static constexpr int NB2 = NB2_;
     static constexpr int LAG = Lag<T, K>::LAG;
     static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
@@ -397,7 +447,7 @@ struct SmemL {
     static constexpr int TMAX = TILE_THREADS * ITEMS;
     static constexpr int NBL = 32;                // look-back binomial rows
     static constexpr int BUFB = ((TMAX * (int)sizeof(T) + 32) + 127) / 128 * 128;
-    static constexpr int WQ = 64 * K;             // per-iteration warp states   [64][K]
+    static constexpr int WQ = (VEC ? 8 : 64) * K; // per-iteration warp states [pairs][K] (VEC: s = 1, 8 warps)
     static constexpr int LA = 8 * K;              // per-iteration tile aggregate [8][K]
     static constexpr int OFF_BUF1 = 0;
     static constexpr int OFF_BUF2 = OFF_BUF1 + NB1 * BUFB;
@@ -412,18 +462,29 @@ struct SmemL {
     static constexpr int OFF_LA = OFF_WQ + NQ * WQ * (int)sizeof(T);     // NQ x [8][K]
     static constexpr int OFF_LP = OFF_LA + NQ * LA * (int)sizeof(T);     // NQ x [8][K] in-super prefix
     static constexpr int OFF_BT = OFF_LP + NQ * LA * (int)sizeof(T);     // [K][32]
-    static constexpr int OFF_BL = OFF_BT + K * 32 * (int)sizeof(T);      // [NBL][K]
-    static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(T);     // [8][K]
-    static constexpr int HOB = 16 + MAXS * K * (int)sizeof(T);           // hand-off entry: i32 r, pad, [MAXS][K]
+    static constexpr int OFF_BN = OFF_BT + K * 32 * (int)sizeof(T);      // [K][32]
+    static constexpr int OFF_BL = OFF_BN + K * 32 * (int)sizeof(T);      // [NBL][K]
+    static constexpr int OFF_BQ = OFF_BL + NBL * K * (int)sizeof(CT);    // [8][K]
+    static constexpr int HOB = 16 + MAXS * K * (int)sizeof(CT);          // hand-off entry: i32 r, pad, [MAXS][K]
     static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
     static constexpr int OFF_PART = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;   // [2][NCARRY][MAXS][K]
-    static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(T);  // [ELAG][TILE_THREADS][K]
+    static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(CT);  // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
 };
-// one carry-application buffer fewer when the larger VEC tiles would not fit
+// one carry-application buffer fewer when the larger VEC tiles would not fit, then one local-scan
+// buffer fewer (large smem-resident pending states)
 template <typename T, int K, bool VEC>
-struct Smem : std::conditional_t<(SmemL<T, K, VEC, Lag<T, K>::NB2>::BYTES <= 227 * 1024),
-                                 SmemL<T, K, VEC, Lag<T, K>::NB2>, SmemL<T, K, VEC, Lag<T, K>::NB2 - 1>> {};
+struct SmemPick {
+    static constexpr int B1 = Lag<T, K>::NB1, B2 = Lag<T, K>::NB2;
+    static constexpr int B2m = B2 - 1 < 2 ? 2 : B2 - 1;
+    using C1 = SmemL<T, K, VEC, B1, B2>;
+    using C2 = SmemL<T, K, VEC, B1, B2m>;
+    using C3 = SmemL<T, K, VEC, B1 - 1, B2m>;
+    static constexpr int LIM = 227 * 1024;
+    using type = std::conditional_t<(C1::BYTES <= LIM), C1, std::conditional_t<(C2::BYTES <= LIM), C2, C3>>;
+};
+template <typename T, int K, bool VEC>
+struct Smem : SmemPick<T, K, VEC>::type {};
 
 // ------------------------------------------------------------------------------------------
 // the kernel
@@ -432,15 +493,19 @@ template <typename T, int K, bool VEC>
 __global__ void __launch_bounds__(Threads<T, K>::VALUE, 1)
 sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     using S = Smem<T, K, VEC>;
+    using CT = typename Coef<T>::type;
     constexpr int ITEMS = S::ITEMS;
     constexpr int NB1 = S::NB1;
     constexpr int NB2 = S::NB2;
     constexpr int NQ = S::NQ;
     constexpr int LAG = S::LAG;
     constexpr bool ESMEM = Lag<T, K>::SMEM;
-    constexpr int PF = Lag<T, K>::PF;
+    constexpr bool EGMEM = Lag<T, K>::GPEND;
+    const int lag = p.lag;
+    constexpr int PF = S::NB1;  // max claimed-but-unscanned tiles
     constexpr int W1 = TagW<T>::W;      // tagged words per published value
     constexpr int V = LB<T, K>::V;
+    constexpr bool TRANSFORM = IsInt<T>::value && K >= 2 && SAM_TRANSFORM;  // integer similarity-transform scans
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(VEC || ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
     static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 4, "ring sizes");
@@ -466,7 +531,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     T* wq_all = (T*)(smem + S::OFF_WQ);
     T* la_all = (T*)(smem + S::OFF_LA);
     T* bt_s = (T*)(smem + S::OFF_BT);
-    T* bl_s = (T*)(smem + S::OFF_BL);
+    T* bn_s = (T*)(smem + S::OFF_BN);
+    CT* bl_s = (CT*)(smem + S::OFF_BL);
     T* bq_s = (T*)(smem + S::OFF_BQ);
 
     const int tid = threadIdx.x;
@@ -506,6 +572,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         *lb_started = -1;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
+    for (int i = tid; i < K * 32; i += blockDim.x) bn_s[i] = (&p.bn[0][0])[i];
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
     for (int i = tid; i < 8 * K; i += blockDim.x) bq_s[i] = (&p.bq[0][0])[i];
     __syncthreads();
@@ -530,7 +597,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     auto wait_or_end = [&](uint64_t* bar, uint32_t par, int it) -> bool {
         bool ended = false;
         while (!mbar_try_wait(bar, par)) {
-            const int end = *sm_end;
+            const int end = flag_ld(sm_end);
             if (end >= 0 && it >= end) { ended = true; break; }
         }
         return !__any_sync(0xffffffffu, ended);
@@ -586,7 +653,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 }
                 // (2) reload (from L2) the next tile whose carry is known, into a free carry buffer
                 if (j2 < j1 && j2 - j3 < NB2 &&
-                    (SAM_EARLY_RELOAD == 2 ? (j2 / p.M <= *lb_started)
+                    (SAM_EARLY_RELOAD == 2 ? (j2 / p.M <= flag_ld(lb_started))
                                            : mbar_test(SAM_EARLY_RELOAD ? &bar_p1[j2 % NQ] : &bar_carry[j2 % NQ],
                                                        (uint32_t)((j2 / NQ) & 1)))) {
                     // groups committed after the store that last used this buffer (iteration j2-NB2)
@@ -604,7 +671,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 // a buffer is free, at most PF tiles are unscanned and a pending-state slot is free
                 // (tile j1's local scan needs the carry application of j1 - LAG done, and a loaded
                 // tile must never wait for that -- its aggregate gates the other CTAs' carries)
-                if (jend < 0 && j1 < j3 + LAG + p.claim_slack &&
+                if (jend < 0 && j1 < j3 + lag + p.claim_slack &&
                     (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
                     (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
                     if (cur_j == cur_cnt) {  // start the next super-tile
@@ -619,7 +686,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                     if (cur_cnt == 0) {
                         jend = j1;
-                        *sm_end = j1;
+                        flag_st(sm_end, j1);
                     } else {
                         const int64_t t = cur_sup * p.M + cur_j;
                         const int qs = j1 % NQ;
@@ -666,6 +733,23 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const bool ok = pair < npair;
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
                 T E[K], yl[K];
+                if constexpr (TRANSFORM) {
+                    // the compute warps left the warp totals Z in the transformed frame: the
+                    // warp aggregate is M(Uw) Z
+                    T zt[K];
+#pragma unroll
+                    for (int t = 0; t < K; ++t) zt[t] = ok ? wq[(qq * s + mm) * K + t] : T(0);
+#pragma unroll
+                    for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                        for (int j = 0; j < t; ++j) zt[t] += p.bw[t - j] * zt[j];
+                    }
+                    if (ok) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = zt[t];
+                    }
+                    __syncwarp();
+                }
                 if constexpr (K < SAM_KS_MIN_K) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) {
@@ -752,11 +836,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if (jsub == cnt - 1) {  // super-tile complete: wake its carry warp (super-tiles round-robin)
                 const int r = i / p.M;
                 // at most one unconsumed phase per barrier: the warp must have taken super-tile r-NCARRY
-                while (cw_taken[r % NCARRY] < r - NCARRY) __nanosleep(32);
+                while (flag_ld(&cw_taken[r % NCARRY]) < r - NCARRY) __nanosleep(32);
                 mbar_arrive(&bar_cw[r % NCARRY]);
             }
             __syncwarp();
-            if (lane == 0) *agg_done = i + 1;
+            if (lane == 0) flag_st(agg_done, i + 1);
         }
     } else if (warp >= NCW + 2) {
         // =========================== carry warps: carry-in of each super-tile ===================
@@ -775,7 +859,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         const bool coop = p.coop != 0;
         const bool lead = !coop || cw == 0;  // finishes the super-tile (hand-off, sub-tile states)
         const int WV = p.Wn * p.Vr;          // super-tiles per window
-        T* const part_s = (T*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
+        CT* const part_s = (CT*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
         for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
             const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
@@ -790,30 +874,30 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 // barrier is never more than one phase ahead and the parity below is unambiguous.
                 mbar_wait(&bar_cw[bw], (uint32_t)((r / NCARRY) & 1));
                 __syncwarp();
-                if (lane == 0) cw_taken[bw] = r;
+                if (lane == 0) flag_st(&cw_taken[bw], r);
             }
             if (lane == 0 && lead) {
                 SAM_TRACE(4, tile * p.M);
-                if (SAM_EARLY_RELOAD == 2) *lb_started = r;  // its tiles may be re-fetched from L2 now
+                if (SAM_EARLY_RELOAD == 2) flag_st(lb_started, r);  // its tiles may be re-fetched from L2 now
             }
 
             SAM_STRESS(2 + cw, tile);
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
-            auto seed_of = [&](int mm, T* out) {
+            auto seed_of = [&](int mm, CT* out) {
                 if (p.seed) {
 #pragma unroll
-                    for (int t = 0; t < K; ++t) out[t] = p.seed[mm * K + t];
+                    for (int t = 0; t < K; ++t) out[t] = CT(p.seed[mm * K + t]);
                     if ((uint64_t)mm < p.h) {
 #pragma unroll
                         for (int t = K - 1; t >= 1; --t) out[t] = out[t] - out[t - 1];
                     }
                 } else {
 #pragma unroll
-                    for (int t = 0; t < K; ++t) out[t] = T(0);
+                    for (int t = 0; t < K; ++t) out[t] = CT(0);
                 }
             };
 
-            T C[K];
+            CT C[K];
             {
                 // lane = (jl, mlb); row vv of window j holds the super-tile at distance
                 // d = j*WV + jl + Wn*vv before S-1; rows beyond Sprev hold nothing, the row AT Sprev
@@ -821,10 +905,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int Wn = p.Wn;
                 const int jl = lane / s, mlb = lane - jl * s;
                 const bool active = jl < Wn;
-                T total[K], Pm[K];
+                CT total[K], Pm[K];
                 const int j0 = coop ? cw : 0, jstep = coop ? NCARRY : 1;
 #pragma unroll
-                for (int t = 0; t < K; ++t) { total[t] = T(0); Pm[t] = p.bwinj[j0][t]; }  // Pm = M(j0 WV US)
+                for (int t = 0; t < K; ++t) { total[t] = CT(0); Pm[t] = p.bwinj[j0][t]; }  // Pm = M(j0 WV US)
                 int npoll = 0;
                 for (int j = j0;; j += jstep) {
                     const int64_t basei = tile - 1 - (int64_t)j * WV;
@@ -881,21 +965,21 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                     // fold.  This lane's rows sit at d = jl + Wn*vv (+ j*WV), so by Horner in vv:
                     //   sum_vv M((jl + Wn vv) US) X_vv = M(jl US) (X_0 + M(Wn US)(X_1 + M(Wn US)(X_2 + ...)))
-                    T Y[K];
+                    CT Y[K];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) Y[t] = T(0);
+                    for (int t = 0; t < K; ++t) Y[t] = CT(0);
 #pragma unroll
                     for (int vv = V - 1; vv >= 0; --vv) {
-                        T X[K];
+                        CT X[K];
 #pragma unroll
-                        for (int t = 0; t < K; ++t) X[t] = T(0);
+                        for (int t = 0; t < K; ++t) X[t] = CT(0);
                         if (st[vv] == 1) {
 #pragma unroll
                             for (int t = 0; t < K; ++t) {
                                 if constexpr (W1 == 1) {
-                                    X[t] = Bits<T>::from(w[vv][t][0] & 0xffffffffull);
+                                    X[t] = CT(Bits<T>::from(w[vv][t][0] & 0xffffffffull));
                                 } else {
-                                    X[t] = Bits<T>::from((w[vv][t][0] & 0xffffffffull) | (w[vv][t][1] << 32));
+                                    X[t] = CT(Bits<T>::from((w[vv][t][0] & 0xffffffffull) | (w[vv][t][1] << 32)));
                                 }
                             }
                         }
@@ -905,7 +989,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         } else {
 #pragma unroll
                             for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn US) Y + X
-                                T acc2 = Y[t] + X[t];
+                                CT acc2 = Y[t] + X[t];
 #pragma unroll
                                 for (int jj = 0; jj < t; ++jj) acc2 += p.bwn[t - jj] * Y[jj];
                                 Y[t] = acc2;
@@ -915,7 +999,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     if (active) {  // Y <- M(jl US) Y
 #pragma unroll
                         for (int t = K - 1; t >= 1; --t) {
-                            T acc2 = Y[t];
+                            CT acc2 = Y[t];
 #pragma unroll
                             for (int jj = 0; jj < t; ++jj) acc2 += bl_s[jl * K + (t - jj)] * Y[jj];
                             Y[t] = acc2;
@@ -924,24 +1008,24 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     for (int off = 1; off < Wn; off <<= 1) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) {
-                            T o = shfl_down(Y[t], off * s);
+                            CT o = shfl_down(Y[t], off * s);
                             if (jl + off < Wn) Y[t] += o;
                         }
                     }
                     // lanes jl == 0 hold this window's sum; total += M(j WV US) Y
 #pragma unroll
                     for (int t = K - 1; t >= 0; --t) {
-                        T acc2 = Y[t];
+                        CT acc2 = Y[t];
 #pragma unroll
                         for (int jj = 0; jj < t; ++jj) acc2 += Pm[t - jj] * Y[jj];
                         total[t] += acc2;
                     }
                     if (last) break;
                     {   // Pm <- Pm * M(jstep*WV*US)  (truncated polynomial product)
-                        T np[K];
+                        CT np[K];
 #pragma unroll
                         for (int d = 0; d < K; ++d) {
-                            T acc2 = T(0);
+                            CT acc2 = CT(0);
 #pragma unroll
                             for (int e2 = 0; e2 <= d; ++e2) acc2 += Pm[e2] * p.bwinj[jstep][d - e2];
                             np[d] = acc2;
@@ -951,7 +1035,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                 }
                 if (coop) {  // sum the warps' partial folds (all already at their absolute offsets)
-                    T* slot = part_s + ((r & 1) * NCARRY + cw) * MAXS * K;
+                    CT* slot = part_s + ((r & 1) * NCARRY + cw) * MAXS * K;
                     if (lane_ok) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) slot[lane * K + t] = total[t];
@@ -960,7 +1044,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     if (lead && lane == 0) SAM_TRACE(13, tile * p.M);
                     if (lead && lane_ok) {
                         for (int w2 = 1; w2 < NCARRY; ++w2) {
-                            const T* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
+                            const CT* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
 #pragma unroll
                             for (int t = 0; t < K; ++t) total[t] += o[lane * K + t];
                         }
@@ -970,25 +1054,25 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     // the CTA's own chain, kept to a few operations: C = F + M((S-1-Sprev) US) I_prev,
                     // I_prev = this CTA's inclusive state after Sprev (hand-off) or, for r = 0, the seed
                     // of virtual super-tile -1 (M(S US) computed here, once per CTA)
-                    T pv[K], bcol[K];
+                    CT pv[K], bcol[K];
                     bool have = false;
                     if (Sprev >= 0) {
                         const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
-                        while (*rt != r - 1) __nanosleep(20);
+                        while (flag_ld_acq(rt) != r - 1) __nanosleep(20);
                         __syncwarp();
-                        const T* hv = (const T*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
+                        const CT* hv = (const CT*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
 #pragma unroll
                         for (int t = 0; t < K; ++t) { pv[t] = hv[ml * K + t]; bcol[t] = p.bprev[t]; }
                         have = true;
                     } else if (p.seed) {
                         seed_of(ml, pv);
-                        mcol<T>(tile * (int64_t)p.M * p.U, K, bcol);
+                        mcol<CT>(tile * (int64_t)p.M * p.U, K, bcol);
                         have = true;
                     }
                     if (have) {
 #pragma unroll
                         for (int t = K - 1; t >= 0; --t) {
-                            T acc2 = total[t] + pv[t];
+                            CT acc2 = total[t] + pv[t];
 #pragma unroll
                             for (int jj = 0; jj < t; ++jj) acc2 += bcol[t - jj] * pv[jj];
                             total[t] = acc2;
@@ -1008,23 +1092,22 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if ((uint64_t)tile + gridDim.x < p.num_super) {
                 if (r > 0) {
                     const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
-                    while (*rt != r - 1) __nanosleep(20);
+                    while (flag_ld_acq(rt) != r - 1) __nanosleep(20);
                 }
                 __syncwarp();
                 unsigned char* ho = smem + S::OFF_HO + (r % NCARRY) * S::HOB;
                 if (lane_ok) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) {
-                        T acc2 = C[t] + la[ml * K + t];
+                        CT acc2 = C[t] + la[ml * K + t];
 #pragma unroll
                         for (int j = 0; j < t; ++j) acc2 += p.bus[t - j] * C[j];
-                        ((T*)(ho + 16))[lane * K + t] = acc2;
+                        ((CT*)(ho + 16))[lane * K + t] = acc2;
                     }
                 }
                 __syncwarp();
                 if (lane == 0) {
-                    __threadfence_block();
-                    *(volatile int*)ho = r;
+                    flag_st_rel((volatile int*)ho, r);
                 }
             }
             if (lane == 0) SAM_TRACE(14, tile * p.M);
@@ -1035,10 +1118,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int qj = (i0 + j) % NQ;
                 T* wq = wq_all + qj * S::WQ;
                 const T* lp = lp_all + qj * S::LA;
-                T Cj[K];
+                CT Cj[K];
 #pragma unroll
                 for (int t = K - 1; t >= 0; --t) {
-                    T acc2 = C[t] + lp[ml * K + t];
+                    CT acc2 = C[t] + lp[ml * K + t];
 #pragma unroll
                     for (int d = 0; d < t; ++d) acc2 += p.bsub[j][t - d] * C[d];
                     Cj[t] = acc2;
@@ -1049,16 +1132,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     const int pair = lane + 32 * ch;
                     const bool ok = pair < npair;
                     const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
-                    T Cm[K];
+                    CT Cm[K];
 #pragma unroll
                     for (int t = 0; t < K; ++t) Cm[t] = shfl_idx(Cj[t], mm);
                     if (ok) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) {
-                            T acc2 = Cm[t] + wq[(qq * s + mm) * K + t];
+                            CT acc2 = Cm[t] + wq[(qq * s + mm) * K + t];
 #pragma unroll
                             for (int d = 0; d < t; ++d) acc2 += bq_s[qq * K + (t - d)] * Cm[d];
-                            wq[(qq * s + mm) * K + t] = acc2;
+                            wq[(qq * s + mm) * K + t] = T(acc2);
                         }
                     }
                 }
@@ -1094,12 +1177,24 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 T Cq[K];
 #pragma unroll
                 for (int t = 0; t < K; ++t) Cq[t] = wq[(q * s + m) * K + t];
+                if constexpr (TRANSFORM) {  // y = M(v ITEMS) (Cq + e'), e' in the transformed frame
+#pragma unroll
+                    for (int t = 0; t < K; ++t) Cq[t] += e[t];
+#pragma unroll
+                    for (int t = 0; t < K; ++t) {
+                        T acc2 = Cq[t];
+#pragma unroll
+                        for (int j = 0; j < t; ++j) acc2 += bt_s[(t - j) * 32 + v] * Cq[j];
+                        y[t] = acc2;
+                    }
+                } else {
 #pragma unroll
                 for (int t = 0; t < K; ++t) {
                     T acc2 = e[t] + Cq[t];
 #pragma unroll
                     for (int j = 0; j < t; ++j) acc2 += bt_s[(t - j) * 32 + v] * Cq[j];
                     y[t] = acc2;
+                }
                 }
             }
             // exclusive: the first K outputs are y_K at positions before the thread's first item,
@@ -1141,21 +1236,14 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     constexpr bool SLOW = decltype(slow_tag)::value;
                     // all ITEMS loads first: interleaving them with the (possibly aliasing, as far
                     // as the compiler knows) stores would serialise every item on an smem round trip
-                    T xv[ITEMS];
+                    // (the slow edge-tile path loads each item where it is used instead: it is cold,
+                    // and holding ITEMS values there only costs registers)
+                    T xv[SLOW ? 1 : ITEMS];
                     if constexpr (VEC && !SLOW) {
                         lds_vec<T, ITEMS>(xs + base_loc, xv);
-                    } else {
+                    } else if constexpr (!SLOW) {
 #pragma unroll
-                    for (int i = 0; i < ITEMS; ++i) {
-                        const int el = base_loc + i * s;
-                        if constexpr (SLOW) {
-                            const uint64_t ve = e0 + el;
-                            const bool valid = !masked || (ve >= p.h && ve < p.h + p.n);
-                            xv[i] = valid ? xs[el] : T(0);
-                        } else {
-                            xv[i] = xs[el];
-                        }
-                    }
+                        for (int i = 0; i < ITEMS; ++i) xv[i] = xs[base_loc + i * s];
                     }
                     T ov[VEC && !SLOW ? ITEMS : 1];
                     if constexpr (VEC && !SLOW && K == 1) {
@@ -1188,21 +1276,29 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         sts_vec<T, ITEMS>(xs + base_loc, ov);
                         return;
                     }
-#pragma unroll
+#pragma unroll(SLOW ? 1 : ITEMS)
                     for (int i = 0; i < ITEMS; ++i) {
                         const int el = base_loc + i * s;
-                        const T x = xv[i];
                         bool valid = true;
                         uint64_t ve = 0;
+                        T x;
                         if constexpr (SLOW) {
                             ve = e0 + el;
                             valid = !masked || (ve >= p.h && ve < p.h + p.n);
+                            x = valid ? xs[el] : T(0);
+                        } else {
+                            x = xv[i];
                         }
                         y[0] += x;
 #pragma unroll
                         for (int t = 1; t < K; ++t) y[t] += y[t - 1];
                         T outv;
-                        if constexpr (EXCL) {  // y_K of item i-K (ring slot i%K), then remember item i
+                        if constexpr (EXCL && SLOW) {  // not unrolled: rotate the ring (static indices)
+                            outv = ring[0];
+#pragma unroll
+                            for (int d = 0; d + 1 < K; ++d) ring[d] = ring[d + 1];
+                            ring[K - 1] = y[K - 1];
+                        } else if constexpr (EXCL) {  // y_K of item i-K (ring slot i%K), then remember item i
                             outv = ring[i % K];
                             ring[i % K] = y[K - 1];
                         } else {
@@ -1298,7 +1394,38 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             //   z_v[t] = a_v[t] + sum_{j<t} b_{t-j}(ITEMS) e_v[j]      (5k dependent shuffle stages)
             // Orders >= 3: Kogge-Stone on k-vectors with the carry operator, level l combining
             //   st <- M(2^l ITEMS) st_partner + st                       (5 dependent stages)
-            if constexpr (K < SAM_KS_MIN_K) {
+            if constexpr (TRANSFORM) {
+                // Integers, orders >= 2: similarity transform.  With z_u = M(-(u+1) ITEMS) a_u,
+                //   e_v = sum_{u<v} M((v-1-u) ITEMS) a_u = M(v ITEMS) sum_{u<v} z_u,
+                // so the k-vector scan becomes K independent plain shuffle scans (depth 5, no
+                // matrix per level); e' = sum_{u<v} z_u is kept and M(v ITEMS) is applied in the
+                // carry application, where it merges with the carry's own M(v ITEMS) (exact mod 2^w).
+                T z[K], Z[K];
+#pragma unroll
+                for (int t = 0; t < K; ++t) {
+                    T acc2 = acc[t];
+#pragma unroll
+                    for (int j = 0; j < t; ++j) acc2 += bn_s[(t - j) * 32 + v] * acc[j];
+                    z[t] = acc2;
+                    Z[t] = acc2;
+                }
+#pragma unroll
+                for (int l = 0; l < 5; ++l) {
+                    const int off = G << l;
+                    if (off < 32) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) {
+                            T o = shfl_up(Z[t], off);
+                            if (lane >= off) Z[t] += o;
+                        }
+                    }
+                }
+#pragma unroll
+                for (int t = 0; t < K; ++t) {
+                    e[t] = Z[t] - z[t];
+                    if (v == Pw - 1) wq[(q * s + m) * K + t] = Z[t];  // transformed warp total of lane m
+                }
+            } else if constexpr (K < SAM_KS_MIN_K) {
 #pragma unroll
                 for (int t = 0; t < K; ++t) {
                     T z = acc[t];
@@ -1361,12 +1488,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 for (int i = 0;; ++i) {
                     const int b1 = i % NB1;
                     if (!wait_or_end(&bar_full1[b1], (uint32_t)((i / NB1) & 1), i)) break;
-                    // the pending-state slot i % LAG must have been consumed by P2 of i - LAG
-                    while (*p2_cnt < (i - LAG + 1) * NW) __nanosleep(32);
+                    // the pending-state slot i % lag must have been consumed by P2 of i - lag
+                    while (flag_ld_acq(p2_cnt) < (i - lag + 1) * NW) __nanosleep(32);
                     T e[K];
                     local_scan(i, b1, e);
 #pragma unroll
-                    for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                    for (int t = 0; t < K; ++t) eq_s[((i % lag) * TILE_THREADS + gtid) * K + t] = e[t];
                 }
             } else {
                 for (int i = 0;; ++i) {
@@ -1375,10 +1502,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                     T e[K];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
+                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % lag) * TILE_THREADS + gtid) * K + t];
                     carry_apply(i, tile_of[i % NQ], e);
                     __syncwarp();
-                    if (lane == 0) atomicAdd((int*)p2_cnt, 1);
+                    if (lane == 0) {
+                        __threadfence_block();  // this warp's reads of its pending states come first
+                        atomicAdd((int*)p2_cnt, 1);
+                    }
                 }
             }
         } else {
@@ -1386,11 +1516,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             // published as early as possible (predecessor aggregates gate every look-back); a
             // tile's carry application (P2) runs once the producer has re-fetched it.  Up to LAG
             // tiles sit between P1 and P2, their local states in registers (static ring eq).
-            T eq[ESMEM ? 1 : LAG][K];  // register ring only when the states do not fit smem
+            T eq[(ESMEM || EGMEM) ? 1 : LAG][K];  // register ring only when the states are in neither smem nor L2
             int p1_next = 0, p2_next = 0;
             for (;;) {
-                const int end = *sm_end;
-                if ((end < 0 || p1_next < end) && p1_next < p2_next + LAG) {
+                const int end = flag_ld(sm_end);
+                if ((end < 0 || p1_next < end) && p1_next < p2_next + lag) {
                     const int i = p1_next;
                     const int b1 = i % NB1;
                     const uint32_t par = (uint32_t)((i / NB1) & 1);
@@ -1399,9 +1529,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         mbar_wait(&bar_full1[b1], par);
                         T e[K];
                         local_scan(i, b1, e);
-                        if constexpr (ESMEM) {
+                        if constexpr (EGMEM) {
+                            T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % lag)) * K * TILE_THREADS + gtid;
 #pragma unroll
-                            for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                            for (int t = 0; t < K; ++t) pe[t * TILE_THREADS] = e[t];
+                        } else if constexpr (ESMEM) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) eq_s[((i % lag) * TILE_THREADS + gtid) * K + t] = e[t];
                         } else {
 #pragma unroll
                             for (int j = 0; j < LAG; ++j) {
@@ -1425,9 +1559,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         mbar_wait(&bar_full2[b2], par);
                         if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                         T e[K];
-                        if constexpr (ESMEM) {
+                        if constexpr (EGMEM) {
+                            const T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % lag)) * K * TILE_THREADS + gtid;
 #pragma unroll
-                            for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
+                            for (int t = 0; t < K; ++t) e[t] = pe[t * TILE_THREADS];
+                        } else if constexpr (ESMEM) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) e[t] = eq_s[((i % lag) * TILE_THREADS + gtid) * K + t];
                         } else {
 #pragma unroll
                             for (int j = 0; j < LAG; ++j) {

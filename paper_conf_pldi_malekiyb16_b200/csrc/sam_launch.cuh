@@ -65,6 +65,7 @@ struct LaunchArgs {
     unsigned long long* trace;
     unsigned long long carry_words;  // capacity of `carry` in 64-bit words (wrap-around reset)
     unsigned int* reset_ctr;         // grid barrier of the epoch wrap-around reset
+    void* pend;                      // pending-state scratch (states > 16 B), pend_bytes() of the workspace
     int num_sms;
     int dev;
 };
@@ -80,6 +81,7 @@ struct Knobs {
     int vr = 0;            // SAM_VR: window rows per round trip
     int coop = -1;         // SAM_COOP: carry warps fold each super-tile together (1) or round-robin (0)
     bool no_vec = false;   // SAM_NO_VEC: never take the 128-bit tuple-1 path
+    int lag = 0;           // SAM_LAG: pipeline depth (tiles between local scan and carry application), <= LAG
 };
 inline const Knobs& knobs() {
     static const Knobs k = [] {
@@ -89,6 +91,7 @@ inline const Knobs& knobs() {
         if (const char* e = getenv("SAM_VR")) r.vr = atoi(e);
         if (const char* e = getenv("SAM_COOP")) r.coop = atoi(e) != 0;
         r.no_vec = getenv("SAM_NO_VEC") != nullptr;
+        if (const char* e = getenv("SAM_LAG")) r.lag = atoi(e);
         return r;
     }();
     return k;
@@ -148,9 +151,20 @@ inline uint32_t& debug_stress() {
     return seed;
 }
 
+// global-memory pending-state scratch of one launch: [grid][LAG][K][TILE_THREADS] elements
+template <typename T, int K>
+constexpr size_t pend_bytes_tk(int num_ctas) {
+    return Lag<T, K>::GPEND ? (size_t)num_ctas * Lag<T, K>::LAG * K * TILE_THREADS * sizeof(T) : 0;
+}
+// upper bound over (element size, order) for the workspace: states > 16 B only
+inline size_t pend_bytes(int w, int k, int num_ctas) {
+    return (SAM_GPEND && w * k > 16) ? (size_t)num_ctas * SAM_LAGG * k * TILE_THREADS * w : 0;
+}
+
 template <typename T, int K, bool VEC>
 cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
     using S = Smem<T, K, VEC>;
+    using CT = typename Coef<T>::type;
     constexpr int ITEMS = Items<T, VEC>::V;
     constexpr int V = LB<T, K>::V;
     static KernelInfo<T, K, VEC> info;
@@ -223,18 +237,20 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
                 mcol<T>(ITEMS, K, t->bc);
                 mcol<T>(geo.Uw, K, t->bw);
                 mcol<T>(geo.U, K, t->bu);
-                mcol<T>(US, K, t->bus);
-                for (int j = 0; j <= NCARRY; ++j) mcol<T>((int64_t)j * geo.Wn * Vr * US, K, t->bwinj[j]);
-                mcol<T>((int64_t)(P - 1) * US, K, t->bprev);
-                mcol<T>((int64_t)geo.Wn * US, K, t->bwn);
+                mcol<CT>(US, K, t->bus);
+                for (int j = 0; j <= NCARRY; ++j) mcol<CT>((int64_t)j * geo.Wn * Vr * US, K, t->bwinj[j]);
+                mcol<CT>((int64_t)(P - 1) * US, K, t->bprev);
+                mcol<CT>((int64_t)geo.Wn * US, K, t->bwn);
                 for (int v = 0; v < 32; ++v) {
                     T b[K];
                     mcol<T>((int64_t)v * ITEMS, K, b);
                     for (int d = 0; d < K; ++d) t->bt[d][v] = b[d];
+                    mcol<T>(-(int64_t)(v + 1) * ITEMS, K, b);
+                    for (int d = 0; d < K; ++d) t->bn[d][v] = b[d];
                 }
                 for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, t->bq[q]);
-                for (int j = 0; j < 32; ++j) mcol<T>((int64_t)j * US, K, t->bl[j]);
-                for (int j = 0; j < 8; ++j) mcol<T>((int64_t)j * geo.U, K, t->bsub[j]);
+                for (int j = 0; j < 32; ++j) mcol<CT>((int64_t)j * US, K, t->bl[j]);
+                for (int j = 0; j < 8; ++j) mcol<CT>((int64_t)j * geo.U, K, t->bsub[j]);
                 for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * ITEMS, K, t->bks[l]);
                 for (int l = 0; l < 3; ++l) mcol<T>((int64_t)(1 << l) * geo.Uw, K, t->bkw[l]);
                 it = tables.emplace(key, t).first;
@@ -268,6 +284,8 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         p.done_ctr = a.done_ctr;
         p.epoch_ptr = a.epoch_ptr;
         p.reset_ctr = a.reset_ctr;
+        p.pend = (T*)a.pend;
+        p.lag = (kn.lag >= 1 && kn.lag <= S::LAG) ? kn.lag : S::LAG;
         p.trace = a.trace;
         p.stress = debug_stress();
 

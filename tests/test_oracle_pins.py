@@ -272,3 +272,16 @@ def test_oracle_rejects_bad_args():
         oracle.scan(np.zeros(4, np.int32), 1, 2, True, phase=2)
     with pytest.raises(ValueError):
         oracle.scan(np.zeros(4, np.int32), 0, 1, True)
+
+
+@pytest.mark.parametrize("name", ["i32", "i64"])
+@pytest.mark.parametrize("k,s", [(1, 1), (3, 1), (2, 5), (8, 8), (4, 3)])
+def test_allcores_context_scan_matches_serial_oracle(name, k, s):
+    """bench.py's all-cores CPU context number runs oracle.scan_allcores (k passes of two-phase
+    order-1 scans over chunks); it must equal the serial oracle bit for bit, for chunk counts that
+    do and do not divide n or s."""
+    x = synth.make(100_003, name, "uniform", seed=k * 10 + s)
+    ref = oracle.scan(x, k, s, True)[0]
+    for threads in (1, 3, 8):
+        got = oracle.scan_allcores(x, k, s, threads=threads)
+        assert np.array_equal(got, ref), f"threads={threads}"

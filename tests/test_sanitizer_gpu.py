@@ -21,10 +21,10 @@ SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitize
 def test_compute_sanitizer(tool):
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not found")
-    cmd = [SAN, "--tool", tool, "--error-exitcode", "97", "--kernel-name", "regex:sam_scan_kernel",
+    cmd = [SAN, "--tool", tool, "--error-exitcode", "97", "--kernel-name", "kns=sam_scan_kernel",
            sys.executable, os.path.join(ROOT, "tests", "sanitize_driver.py")]
     if tool == "racecheck":
-        cmd[3:3] = ["--racecheck-report", "hazard"]
+        cmd[3:3] = ["--racecheck-report", "hazard", "--print-limit", "400"]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=3000, cwd=ROOT)
     out = r.stdout + r.stderr
     with open(os.path.join(ROOT, "gpurun_out", f"sanitizer_{tool}.txt") if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else os.devnull, "w") as f:
