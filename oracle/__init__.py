@@ -87,6 +87,11 @@ def _load():
             fn = getattr(lib, name)
             fn.argtypes = [P, ctypes.c_uint64, ctypes.c_int, ctypes.c_int]
             fn.restype = ctypes.c_int
+        for name in ("oracle_scan_op_i32", "oracle_scan_op_u32", "oracle_scan_op_i64", "oracle_scan_op_u64",
+                     "oracle_scan_op_f32", "oracle_scan_op_f64"):
+            fn = getattr(lib, name)
+            fn.argtypes = [P, ctypes.c_uint64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, P]
+            fn.restype = ctypes.c_int
         lib.oracle_sizeof_long_double.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -149,6 +154,45 @@ def delta(x: np.ndarray, k: int, s: int = 1) -> np.ndarray:
     if rc != 0:
         raise ValueError(f"oracle rejected arguments (rc={rc}): k={k} s={s}")
     return a
+
+
+OPS = {"add": 0, "xor": 1, "max": 2, "min": 3}
+_OP_FN = {np.dtype(np.int32): "i32", np.dtype(np.uint32): "u32", np.dtype(np.int64): "i64",
+          np.dtype(np.uint64): "u64", np.dtype(np.float32): "f32", np.dtype(np.float64): "f64"}
+
+
+def op_identity(op: str, dtype):
+    """Identity element of `op` on dtype (reading R14): xor 0; max: lowest value (-inf for
+    floats); min: highest value (+inf for floats)."""
+    dt = np.dtype(dtype)
+    if op == "xor":
+        return dt.type(0)
+    if dt.kind == "f":
+        return dt.type(-np.inf if op == "max" else np.inf)
+    info = np.iinfo(dt)
+    return dt.type(info.min if op == "max" else info.max)
+
+
+def scan_op(x: np.ndarray, op: str, k: int, s: int = 1, inclusive: bool = True, phase: int = 0, run=None):
+    """Order-k, tuple-s scan of x under `op` in {"xor", "max", "min"} (sam_oracle.c
+    oracle_scan_op_*): the serial loop with op in place of +, in the element type.  Returns (y, run).
+    ("add" is scan().)"""
+    lib = _load()
+    x = np.ascontiguousarray(x)
+    if op not in ("xor", "max", "min"):
+        raise ValueError("scan_op: op must be xor, max or min (add is oracle.scan)")
+    if op == "xor" and x.dtype.kind == "f":
+        raise ValueError("xor is defined for integers only")
+    a = x.copy()
+    if run is None:
+        run = np.full(k * s, op_identity(op, x.dtype), dtype=x.dtype)
+    else:
+        run = np.ascontiguousarray(run, dtype=x.dtype)
+    fn = getattr(lib, "oracle_scan_op_" + _OP_FN[x.dtype])
+    rc = fn(a.ctypes.data, a.size, OPS[op], int(k), int(s), int(bool(inclusive)), int(phase), run.ctypes.data)
+    if rc != 0:
+        raise ValueError(f"oracle rejected arguments (rc={rc})")
+    return a, run
 
 
 def long_double_bytes() -> int:

@@ -148,7 +148,7 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #define SAM_GPEND 1
 #endif
 #ifndef SAM_LAGG
-#define SAM_LAGG 12
+#define SAM_LAGG 8
 #endif
 // states of 33..64 B (int64 orders 5-8) without SAM_GPEND: pending in shared memory, LAG 4
 #ifndef SAM_SMEM64
@@ -246,6 +246,7 @@ struct Params {
     T bt[K][32];          // b_d(v*ITEMS),  v < Pw        ([d][v])
     T bn[K][32];          // b_d(-(v+1)*ITEMS), v < Pw    ([d][v]; integer similarity transform)
     T bq[8][K];           // b_d(q*Uw),     q < c
+    T bqn[8][K];          // b_d(-q*Uw),    q < c         (integer similarity transform)
     CT bl[32][K];         // b_d(j*M*U),    j < Wn
     CT bsub[8][K];        // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
     T bks[5][K];          // b_d(2^l*ITEMS) (Kogge-Stone warp scan of thread states, K >= 3)
@@ -356,24 +357,19 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-// CTA-scope flags in shared memory (end-of-stream, progress counters, hand-off stamps): relaxed
-// atomic accesses (morally strong in the PTX memory model, and visible as such to racecheck), the
-// data they guard ordered by fences (writer: fence before the flag; reader: flag before the data)
-__device__ __forceinline__ int flag_ld(const volatile int* p) {
-    int v;
-    asm volatile("ld.relaxed.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32((const void*)p)) : "memory");
-    return v;
-}
+// CTA-scope flags in shared memory (end-of-stream, progress counters, hand-off stamps): atomic
+// accesses (racecheck treats them as synchronisation; they sit only on wait paths), the data they
+// guard ordered by CTA fences (writer: fence, then the flag; reader: the flag, then a fence)
+__device__ __forceinline__ int flag_ld(const volatile int* p) { return atomicOr((int*)p, 0); }
 __device__ __forceinline__ int flag_ld_acq(const volatile int* p) {
-    int v;
-    asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32((const void*)p)) : "memory");
+    const int v = atomicOr((int*)p, 0);
+    __threadfence_block();
     return v;
 }
+__device__ __forceinline__ void flag_st(volatile int* p, int v) { atomicExch((int*)p, v); }
 __device__ __forceinline__ void flag_st_rel(volatile int* p, int v) {
-    asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_u32((const void*)p)), "r"(v) : "memory");
-}
-__device__ __forceinline__ void flag_st(volatile int* p, int v) {
-    asm volatile("st.relaxed.cta.shared.b32 [%0], %1;" ::"r"(smem_u32((const void*)p)), "r"(v) : "memory");
+    __threadfence_block();
+    atomicExch((int*)p, v);
 }
 __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
     unsigned long long a;
@@ -452,7 +448,7 @@ struct SmemL {
     static constexpr int OFF_BUF1 = 0;
     static constexpr int OFF_BUF2 = OFF_BUF1 + NB1 * BUFB;
     static constexpr int OFF_BAR = OFF_BUF2 + NB2 * BUFB;  // full1[NB1] full2[NB2] stored2[NB2] p1/agg/carry[NQ]
-    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ + NCARRY;
+    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ + NCARRY + 1;  // ... bar_cw[NCARRY], bar_land
     static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
     static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
     static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
@@ -469,7 +465,13 @@ struct SmemL {
     static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
     static constexpr int OFF_PART = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;   // [2][NCARRY][MAXS][K]
     static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(CT);  // [ELAG][TILE_THREADS][K]
-    static constexpr int BYTES = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
+    static constexpr int BYTES0 = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
+    // carry-fold landing buffer: the P-1 aggregates a fold reads, pulled from L2 in ONE bulk copy
+    // (whatever shared memory is left, up to 40 KB; the fold falls back to windowed loads if short)
+    static constexpr int OFF_LAND = (BYTES0 + 127) / 128 * 128;
+    static constexpr int LAND_ROOM = 227 * 1024 - OFF_LAND;
+    static constexpr int LANDB = LAND_ROOM < 0 ? 0 : (LAND_ROOM > 40960 ? 40960 : LAND_ROOM / 128 * 128);
+    static constexpr int BYTES = OFF_LAND + LANDB;
 };
 // one carry-application buffer fewer when the larger VEC tiles would not fit, then one local-scan
 // buffer fewer (large smem-resident pending states)
@@ -481,7 +483,7 @@ struct SmemPick {
     using C2 = SmemL<T, K, VEC, B1, B2m>;
     using C3 = SmemL<T, K, VEC, B1 - 1, B2m>;
     static constexpr int LIM = 227 * 1024;
-    using type = std::conditional_t<(C1::BYTES <= LIM), C1, std::conditional_t<(C2::BYTES <= LIM), C2, C3>>;
+    using type = std::conditional_t<(C1::BYTES0 <= LIM), C1, std::conditional_t<(C2::BYTES0 <= LIM), C2, C3>>;
 };
 template <typename T, int K, bool VEC>
 struct Smem : SmemPick<T, K, VEC>::type {};
@@ -519,6 +521,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint64_t* bar_agg = bar_p1 + NQ;
     uint64_t* bar_carry = bar_agg + NQ;
     uint64_t* bar_cw = bar_carry + NQ;  // [NCARRY]: a super-tile is ready for carry warp w
+    uint64_t* bar_land = bar_cw + NCARRY;  // the fold's landing buffer is full
     volatile int* cw_taken = (volatile int*)(smem + S::OFF_CW);  // last super-tile each carry warp took
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
     int64_t* sup_of = (int64_t*)(smem + S::OFF_SUP);
@@ -558,6 +561,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         }
         for (int w = 0; w < NCARRY; ++w) {
             mbar_init(&bar_cw[w], 32);
+            if (w == 0) mbar_init(bar_land, 1);
             cw_taken[w] = -1;
             *(volatile int*)(smem + S::OFF_HO + w * S::HOB) = -1;
         }
@@ -734,23 +738,39 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int mm = ok ? (pair >> p.logc) : 0, qq = pair & (c - 1);
                 T E[K], yl[K];
                 if constexpr (TRANSFORM) {
-                    // the compute warps left the warp totals Z in the transformed frame: the
-                    // warp aggregate is M(Uw) Z
-                    T zt[K];
+                    // Integers: the compute warps left each warp's total Z_q in its transformed frame
+                    // (warp aggregate A_q = M(Uw) Z_q).  With z'_q = M(-q Uw) Z_q,
+                    //   E_q = sum_{p<q} M((q-1-p) Uw) A_p = M(q Uw) sum_{p<q} z'_p,
+                    // so the combine is K plain scans over the c warps; E'_q = sum_{p<q} z'_p is
+                    // stored (the carry team applies M(q Uw) with its own), and the tile aggregate
+                    // is M(U) (sum of all z'), folded into the running prefix as M(U)(Pref + sum).
+                    T zq[K];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) zt[t] = ok ? wq[(qq * s + mm) * K + t] : T(0);
+                    for (int t = 0; t < K; ++t) {
+                        T acc2 = ok ? wq[(qq * s + mm) * K + t] : T(0);
+                        yl[t] = acc2;
+                    }
 #pragma unroll
                     for (int t = K - 1; t >= 1; --t) {
 #pragma unroll
-                        for (int j = 0; j < t; ++j) zt[t] += p.bw[t - j] * zt[j];
+                        for (int j = 0; j < t; ++j) yl[t] += p.bqn[qq][t - j] * yl[j];
                     }
-                    if (ok) {
 #pragma unroll
-                        for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = zt[t];
+                    for (int t = 0; t < K; ++t) zq[t] = yl[t];
+#pragma unroll
+                    for (int l = 0; l < 3; ++l) {  // offsets 1, 2, 4 < c
+                        const int off = 1 << l;
+                        if (off < c) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) {
+                                T o = shfl_up(yl[t], off);
+                                if (qq >= off) yl[t] += o;
+                            }
+                        }
                     }
-                    __syncwarp();
-                }
-                if constexpr (K < SAM_KS_MIN_K) {
+#pragma unroll
+                    for (int t = 0; t < K; ++t) E[t] = yl[t] - zq[t];  // E'_q; yl = inclusive sum
+                } else                 if constexpr (K < SAM_KS_MIN_K) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) {
                         T z = ok ? wq[(qq * s + mm) * K + t] : T(0);
@@ -811,12 +831,22 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
 #pragma unroll
                         for (int t = 0; t < K; ++t) lp[mm * K + t] = Pref[ch][t];  // state before sub-tile
+                        if constexpr (TRANSFORM) {  // Pref <- M(U) (Pref + sum z')
+#pragma unroll
+                            for (int t = 0; t < K; ++t) Pref[ch][t] += yl[t];
+#pragma unroll
+                            for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                                for (int j = 0; j < t; ++j) Pref[ch][t] += p.bu[t - j] * Pref[ch][j];
+                            }
+                        } else {
 #pragma unroll
                         for (int t = K - 1; t >= 0; --t) {  // Pref <- M(U) Pref + A_j
                             T acc2 = Pref[ch][t] + yl[t];
 #pragma unroll
                             for (int j = 0; j < t; ++j) acc2 += p.bu[t - j] * Pref[ch][j];
                             Pref[ch][t] = acc2;
+                        }
                         }
                         if (jsub == cnt - 1) {
 #pragma unroll
@@ -860,6 +890,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         const bool lead = !coop || cw == 0;  // finishes the super-tile (hand-off, sub-tile states)
         const int WV = p.Wn * p.Vr;          // super-tiles per window
         CT* const part_s = (CT*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
+        // landing: the whole range of aggregates a fold reads (at most P-1 super-tiles of s*K values)
+        // arrives in shared memory with one bulk copy; words whose tag is not yet this launch's are
+        // re-polled from L2 (the nearest predecessors, published last)
+        constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
+        const bool use_land = coop && S::LANDB > 0 &&
+                              (uint64_t)(gridDim.x - 1) * s * SUPB + 32 <= (uint64_t)S::LANDB;
+        int nland = 0;  // landing copies consumed so far (mbarrier parity)
         for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
             const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
@@ -868,6 +905,19 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
             const int bw = coop ? (int)(r % NCARRY) : cw;  // the aggregator's barrier for super-tile r
+            // landing range [lo_sup, tile) in bytes, 16-B aligned.  The copy is issued before the wait
+            // for this super-tile's own aggregate: the previous round's aggregates are long published,
+            // the current round's (the nearest) are re-polled from L2 if not yet there.
+            const int64_t lo_sup = Sprev + 1;
+            const bool land_r = use_land && tile > lo_sup;
+            const uintptr_t land_a16 = ((uintptr_t)p.carry + (uintptr_t)lo_sup * s * SUPB) & ~(uintptr_t)15;
+            if (land_r && lead && lane == 0) {
+                const uintptr_t b16 = ((uintptr_t)p.carry + (uintptr_t)tile * s * SUPB + 15) & ~(uintptr_t)15;
+                fence_proxy_async_smem();  // the previous fold's generic reads of the buffer come first
+                mbar_arrive_expect_tx(bar_land, (uint32_t)(b16 - land_a16));
+                bulk_g2s(smem + S::OFF_LAND, (const void*)land_a16, (uint32_t)(b16 - land_a16), bar_land,
+                         policy_evict_last());
+            }
             if (lead) {
                 // Wait for the aggregator: it arrives on bar_cw[r % NCARRY] when super-tile r is
                 // fully aggregated, and only after super-tile r - NCARRY was taken (cw_taken), so the
@@ -882,6 +932,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             }
 
             SAM_STRESS(2 + cw, tile);
+            if (land_r) {
+                mbar_wait(bar_land, (uint32_t)(nland & 1));
+                ++nland;
+            }
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
             auto seed_of = [&](int mm, CT* out) {
                 if (p.seed) {
@@ -920,6 +974,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         const int64_t idx = basei - jl - (int64_t)Wn * vv;
                         st[vv] = (!active || vv >= p.Vr || idx <= Sprev) ? 3 : 0;
                     }
+                    bool from_land = land_r;  // first pass from the landing buffer, re-polls from L2
                     for (;;) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
                         // all loads first, then the tag checks: the loads of a window are then in
@@ -929,6 +984,15 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             if (st[vv] == 0) {
                                 const int64_t idx = basei - jl - (int64_t)Wn * vv;
                                 const unsigned long long* src = p.carry + ((size_t)idx * s + mlb) * K * W1;
+                                if (from_land) {
+                                    const unsigned long long* ls = (const unsigned long long*)(
+                                        smem + S::OFF_LAND + ((uintptr_t)src - land_a16));
+#pragma unroll
+                                    for (int t = 0; t < K; ++t) {
+#pragma unroll
+                                        for (int h = 0; h < W1; ++h) w[vv][t][h] = ls[t * W1 + h];
+                                    }
+                                } else {
 #pragma unroll
                                 for (int t = 0; t < K; ++t) {
                                     if constexpr (W1 == 1) {
@@ -937,8 +1001,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                         ld_relaxed_v2(src + 2 * t, w[vv][t][0], w[vv][t][1]);
                                     }
                                 }
+                                }
                             }
                         }
+                        from_land = false;
                         bool pend = false;
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
@@ -1117,7 +1183,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             for (int j = 0; j < cnt; ++j) {
                 const int qj = (i0 + j) % NQ;
                 T* wq = wq_all + qj * S::WQ;
-                const T* lp = lp_all + qj * S::LA;
+                T* lp = lp_all + qj * S::LA;
                 CT Cj[K];
 #pragma unroll
                 for (int t = K - 1; t >= 0; --t) {
@@ -1126,8 +1192,18 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     for (int d = 0; d < t; ++d) acc2 += p.bsub[j][t - d] * C[d];
                     Cj[t] = acc2;
                 }
+                if constexpr (TRANSFORM) {
+                    // integers: the sub-tile's carry C_j per lane goes to the compute threads, which
+                    // form M(q Uw) (C_j + E'_q) themselves (no per-warp pass on this serial path)
+                    __syncwarp();
+                    if (lane_ok) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) lp[ml * K + t] = T(Cj[t]);
+                    }
+                }
 #pragma unroll
                 for (int ch = 0; ch < 2; ++ch) {
+                    if constexpr (TRANSFORM) break;
                     if (32 * ch >= npair) break;  // warp-uniform: second pass only for s = 8
                     const int pair = lane + 32 * ch;
                     const bool ok = pair < npair;
@@ -1136,12 +1212,24 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                     for (int t = 0; t < K; ++t) Cm[t] = shfl_idx(Cj[t], mm);
                     if (ok) {
+                        if constexpr (TRANSFORM) {  // M(q Uw) (C_m + E'_q)
+#pragma unroll
+                            for (int t = 0; t < K; ++t) Cm[t] += wq[(qq * s + mm) * K + t];
+#pragma unroll
+                            for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                                for (int d = 0; d < t; ++d) Cm[t] += bq_s[qq * K + (t - d)] * Cm[d];
+                            }
+#pragma unroll
+                            for (int t = 0; t < K; ++t) wq[(qq * s + mm) * K + t] = T(Cm[t]);
+                        } else {
 #pragma unroll
                         for (int t = 0; t < K; ++t) {
                             CT acc2 = Cm[t] + wq[(qq * s + mm) * K + t];
 #pragma unroll
                             for (int d = 0; d < t; ++d) acc2 += bq_s[qq * K + (t - d)] * Cm[d];
                             wq[(qq * s + mm) * K + t] = T(acc2);
+                        }
                         }
                     }
                 }
@@ -1177,7 +1265,15 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 T Cq[K];
 #pragma unroll
                 for (int t = 0; t < K; ++t) Cq[t] = wq[(q * s + m) * K + t];
-                if constexpr (TRANSFORM) {  // y = M(v ITEMS) (Cq + e'), e' in the transformed frame
+                if constexpr (TRANSFORM) {  // y = M(v ITEMS) (M(q Uw) (C_j + E'_q) + e')
+                    const T* cj = lp_all + qs * S::LA;  // the sub-tile's carry, lane m
+#pragma unroll
+                    for (int t = 0; t < K; ++t) Cq[t] += cj[m * K + t];
+#pragma unroll
+                    for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                        for (int d = 0; d < t; ++d) Cq[t] += bq_s[q * K + (t - d)] * Cq[d];
+                    }
 #pragma unroll
                     for (int t = 0; t < K; ++t) Cq[t] += e[t];
 #pragma unroll
@@ -1493,7 +1589,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     T e[K];
                     local_scan(i, b1, e);
 #pragma unroll
-                    for (int t = 0; t < K; ++t) eq_s[((i % lag) * TILE_THREADS + gtid) * K + t] = e[t];
+                    for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
                 }
             } else {
                 for (int i = 0;; ++i) {
@@ -1502,7 +1598,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                     T e[K];
 #pragma unroll
-                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % lag) * TILE_THREADS + gtid) * K + t];
+                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
                     carry_apply(i, tile_of[i % NQ], e);
                     __syncwarp();
                     if (lane == 0) {
@@ -1518,8 +1614,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             // tiles sit between P1 and P2, their local states in registers (static ring eq).
             T eq[(ESMEM || EGMEM) ? 1 : LAG][K];  // register ring only when the states are in neither smem nor L2
             int p1_next = 0, p2_next = 0;
+            int end = -1;  // end-of-stream iteration, refreshed only when idle
             for (;;) {
-                const int end = flag_ld(sm_end);
                 if ((end < 0 || p1_next < end) && p1_next < p2_next + lag) {
                     const int i = p1_next;
                     const int b1 = i % NB1;
@@ -1530,12 +1626,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         T e[K];
                         local_scan(i, b1, e);
                         if constexpr (EGMEM) {
-                            T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % lag)) * K * TILE_THREADS + gtid;
+                            T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % LAG)) * K * TILE_THREADS + gtid;
 #pragma unroll
                             for (int t = 0; t < K; ++t) pe[t * TILE_THREADS] = e[t];
                         } else if constexpr (ESMEM) {
 #pragma unroll
-                            for (int t = 0; t < K; ++t) eq_s[((i % lag) * TILE_THREADS + gtid) * K + t] = e[t];
+                            for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
                         } else {
 #pragma unroll
                             for (int j = 0; j < LAG; ++j) {
@@ -1560,12 +1656,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                         T e[K];
                         if constexpr (EGMEM) {
-                            const T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % lag)) * K * TILE_THREADS + gtid;
+                            const T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % LAG)) * K * TILE_THREADS + gtid;
 #pragma unroll
                             for (int t = 0; t < K; ++t) e[t] = pe[t * TILE_THREADS];
                         } else if constexpr (ESMEM) {
 #pragma unroll
-                            for (int t = 0; t < K; ++t) e[t] = eq_s[((i % lag) * TILE_THREADS + gtid) * K + t];
+                            for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
                         } else {
 #pragma unroll
                             for (int j = 0; j < LAG; ++j) {
@@ -1582,6 +1678,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 } else if (end >= 0 && p1_next >= end) {
                     break;
                 }
+                // warp-uniform refresh: one atomic read, broadcast (per-lane atomics could see
+                // different values and split the warp's control flow)
+                end = __shfl_sync(0xffffffffu, lane == 0 ? flag_ld(sm_end) : 0, 0);
                 __nanosleep(SAM_IDLE_NS);  // nothing ready: yield issue slots to the other warps
             }
         }

@@ -249,6 +249,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
                     for (int d = 0; d < K; ++d) t->bn[d][v] = b[d];
                 }
                 for (int q = 0; q < 8; ++q) mcol<T>((int64_t)q * geo.Uw, K, t->bq[q]);
+                for (int q = 0; q < 8; ++q) mcol<T>(-(int64_t)q * geo.Uw, K, t->bqn[q]);
                 for (int j = 0; j < 32; ++j) mcol<CT>((int64_t)j * US, K, t->bl[j]);
                 for (int j = 0; j < 8; ++j) mcol<CT>((int64_t)j * geo.U, K, t->bsub[j]);
                 for (int l = 0; l < 5; ++l) mcol<T>((int64_t)(1 << l) * ITEMS, K, t->bks[l]);
