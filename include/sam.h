@@ -56,7 +56,19 @@
 extern "C" {
 #endif
 
-typedef enum { SAM_I32 = 0, SAM_I64 = 1, SAM_F32 = 2, SAM_F64 = 3 } sam_dtype;
+/* SAM_U32 / SAM_U64: unsigned integers -- the same bits as SAM_I32 / SAM_I64 for add and xor, and the
+ * unsigned order for max / min (SAM_I32 / SAM_I64 are signed there). */
+typedef enum { SAM_I32 = 0, SAM_I64 = 1, SAM_F32 = 2, SAM_F64 = 3, SAM_U32 = 4, SAM_U64 = 5 } sam_dtype;
+
+/* Associative operators ("prefix scans"). */
+typedef enum { SAM_OP_ADD = 0, SAM_OP_XOR = 1, SAM_OP_MAX = 2, SAM_OP_MIN = 3 } sam_op;
+
+/* Inter-tile carry schemes (the paper's Sec. 5.4). */
+typedef enum {
+    SAM_CARRY_STATIC = 0,   /* SAM's persistent-block schedule, P:783-832 (cooperative grid) */
+    SAM_CARRY_LOOKBACK = 1, /* decoupled look-back over dynamically claimed tiles (no co-residency) */
+    SAM_CARRY_CHAINED = 2   /* each tile waits for its predecessor's inclusive state */
+} sam_carry;
 
 typedef enum {
     SAM_OK = 0,
@@ -187,6 +199,32 @@ int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in,
  * SAM_ERR_INVALID_ARG. */
 int sam_delta_encode_host(sam_dtype dtype, int order, int tuple, const void* in_host, void* out_host,
                           uint64_t n, sam_stream_t stream);
+
+/*
+ * sam_scan_op -- order-k, tuple-s scan under operator `op` (NEXT-4).
+ *   SAM_OP_ADD  = sam_scan (the production single-pass kernel).
+ *   SAM_OP_XOR  integers only (floats -> SAM_ERR_UNSUPPORTED): addition in GF(2)^w, so the order-k
+ *               carry algebra is the additive one with binomials reduced mod 2.
+ *   SAM_OP_MAX / SAM_OP_MIN: every dtype; signed or unsigned order by dtype; floats use IEEE
+ *               maxNum/minNum (a NaN operand is ignored; an all-NaN prefix yields the identity).
+ *               Idempotent, so order k inclusive = order 1, and order k exclusive = the inclusive
+ *               scan shifted by k lane positions (identity -inf/+inf/INT_MIN/... in front).
+ *   Exclusive (all ops): the order-1 exclusive operator applied k times (reading R1), identity-seeded.
+ *   Runs the generic kernel (sam_generic.cuh) with SAM's static carry schedule, falling back to the
+ *   look-back form when no cooperative grid can form.  Arguments as sam_scan.
+ */
+int sam_scan_op(sam_dtype dtype, sam_op op, int order, int tuple, int inclusive, const void* in,
+                void* out, uint64_t n, sam_stream_t stream);
+
+/*
+ * sam_scan_generic -- the generic kernel with an explicit carry scheme (NEXT-3 ablation: the same
+ * intra-tile code under SAM's static schedule, decoupled look-back, or the chained scheme; the
+ * look-back and chained forms need no co-resident grid).  `op` as sam_scan_op (ADD included).
+ * sam_last_carry_scheme() returns the scheme the last call on this thread actually ran.
+ */
+int sam_scan_generic(sam_dtype dtype, sam_op op, sam_carry carry, int order, int tuple, int inclusive,
+                     const void* in, void* out, uint64_t n, sam_stream_t stream);
+int sam_last_carry_scheme(void);
 
 /* Diagnostics */
 const char* sam_last_error(void);

@@ -16,12 +16,15 @@ import os
 __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
     "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_scan_workspace_size", "sam_scan_ws",
-    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_shard_payload_bytes",
+    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_scan_op", "sam_scan_generic", "sam_last_carry_scheme",
+    "scan_op", "SAM_U32", "SAM_U64", "SAM_OP", "SAM_CARRY", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
     "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "sam_delta_encode_host", "delta_encode_host", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
 ]
 
-SAM_I32, SAM_I64, SAM_F32, SAM_F64 = 0, 1, 2, 3
+SAM_I32, SAM_I64, SAM_F32, SAM_F64, SAM_U32, SAM_U64 = 0, 1, 2, 3, 4, 5
+SAM_OP = {"add": 0, "xor": 1, "max": 2, "min": 3}
+SAM_CARRY = {"static": 0, "lookback": 1, "chained": 2}
 _STATUS = {0: "SAM_OK", -1: "SAM_ERR_INVALID_ARG", -2: "SAM_ERR_UNSUPPORTED", -3: "SAM_ERR_CUDA",
            -4: "SAM_ERR_OOM", -5: "SAM_ERR_INTERNAL"}
 
@@ -63,6 +66,9 @@ def lib() -> ctypes.CDLL:
             "sam_launch_count": (U64, []),
             "sam_debug_set_trace": (I, [P]),
             "sam_debug_limit_grid": (I, [U64]),
+            "sam_scan_op": (I, [I, I, I, I, I, P, P, U64, P]),
+            "sam_scan_generic": (I, [I, I, I, I, I, I, P, P, U64, P]),
+            "sam_last_carry_scheme": (I, []),
             "sam_debug_set_stress": (I, [ctypes.c_uint32]),
             "sam_scan_workspace_size": (I, [I, I, I, U64, ctypes.POINTER(SZ)]),
             "sam_scan_ws": (I, [I, I, I, I, P, P, U64, P, SZ, P]),
@@ -106,6 +112,19 @@ def sam_scan_workspace_size(dtype, order, tuple_, n) -> int:
 def sam_scan_ws(dtype, order, tuple_, inclusive, in_ptr, out_ptr, n, ws_ptr, ws_bytes, stream=None) -> int:
     return _check(lib().sam_scan_ws(dtype, order, tuple_, int(bool(inclusive)), in_ptr, out_ptr, n, ws_ptr,
                                     ws_bytes, stream))
+
+
+def sam_scan_op(dtype, op, order, tuple_, inclusive, in_ptr, out_ptr, n, stream=None) -> int:
+    return _check(lib().sam_scan_op(dtype, op, order, tuple_, int(bool(inclusive)), in_ptr, out_ptr, n, stream))
+
+
+def sam_scan_generic(dtype, op, carry, order, tuple_, inclusive, in_ptr, out_ptr, n, stream=None) -> int:
+    return _check(lib().sam_scan_generic(dtype, op, carry, order, tuple_, int(bool(inclusive)), in_ptr, out_ptr, n,
+                                         stream))
+
+
+def sam_last_carry_scheme() -> int:
+    return int(lib().sam_last_carry_scheme())
 
 
 def sam_debug_limit_grid(max_ctas: int) -> int:
@@ -171,6 +190,9 @@ def dtype_code(dt) -> int:
     import torch
 
     m = {torch.int32: SAM_I32, torch.int64: SAM_I64, torch.float32: SAM_F32, torch.float64: SAM_F64}
+    for name, code in (("uint32", SAM_U32), ("uint64", SAM_U64)):
+        if hasattr(torch, name):
+            m[getattr(torch, name)] = code
     if dt not in m:
         raise SamError(-2, f"unsupported dtype {dt} (int32, int64, float32, float64)")
     return m[dt]
@@ -196,6 +218,31 @@ def scan(x, order: int = 1, tuple: int = 1, inclusive: bool = True, out=None, st
         out = torch.empty_like(x)
     sam_scan(dtype_code(x.dtype), order, tuple, inclusive, ctypes.c_void_p(x.data_ptr()),
              ctypes.c_void_p(out.data_ptr()), x.numel(), _stream_ptr(stream))
+    return out
+
+
+def scan_op(x, op: str = "add", order: int = 1, tuple: int = 1, inclusive: bool = True, out=None, stream=None,
+            carry: str | None = None):
+    """Order-`order`, tuple-`tuple` scan of a 1-D contiguous CUDA tensor under `op` in
+    {"add", "xor", "max", "min"} (sam_scan_op; P:367-379).  `carry` in {"static", "lookback",
+    "chained"} selects the generic kernel's carry scheme explicitly (sam_scan_generic, the NEXT-3
+    ablation); None = the library's default path for the operator."""
+    if not x.is_cuda or x.dim() != 1 or not x.is_contiguous():
+        raise SamError(-1, "scan_op() needs a 1-D contiguous CUDA tensor")
+    if op not in SAM_OP:
+        raise SamError(-2, f"unknown operator {op!r}")
+    if out is None:
+        import torch
+
+        out = torch.empty_like(x)
+    args = (order, tuple, inclusive, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()), x.numel(),
+            _stream_ptr(stream))
+    if carry is None:
+        sam_scan_op(dtype_code(x.dtype), SAM_OP[op], *args)
+    else:
+        if carry not in SAM_CARRY:
+            raise SamError(-2, f"unknown carry scheme {carry!r}")
+        sam_scan_generic(dtype_code(x.dtype), SAM_OP[op], SAM_CARRY[carry], *args)
     return out
 
 

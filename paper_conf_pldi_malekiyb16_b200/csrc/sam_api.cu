@@ -14,6 +14,7 @@
 #include <utility>
 
 #include "sam.h"
+#include "sam_generic_launch.h"
 #include "sam_launch.cuh"
 
 namespace sam {
@@ -27,6 +28,7 @@ template <typename T> cudaError_t launch_payload_init(void*, uint64_t, uint64_t,
 namespace {
 
 thread_local std::string g_err;
+thread_local int g_last_carry = -1;  // carry scheme the last generic launch on this thread ran
 std::atomic<uint64_t> g_launches{0};
 constexpr const char* kVersion = "sam-b200 0.2 (sm_100a, single-pass, SAM static carry schedule on a cooperative persistent grid, order 1-8, tuple 1-8)";
 
@@ -39,10 +41,13 @@ int cuda_fail(cudaError_t e, const char* where) {
     return SAM_ERR_CUDA;
 }
 
-size_t elem_size(sam_dtype d) { return (d == SAM_I32 || d == SAM_F32) ? 4 : 8; }
+size_t elem_size(sam_dtype d) { return (d == SAM_I32 || d == SAM_F32 || d == SAM_U32) ? 4 : 8; }
+
+// SAM_U32 / SAM_U64 are the same bits as SAM_I32 / SAM_I64 for addition (wraparound)
+sam_dtype add_dtype(sam_dtype d) { return d == SAM_U32 ? SAM_I32 : (d == SAM_U64 ? SAM_I64 : d); }
 
 int validate_common(sam_dtype dtype, int order, int tuple) {
-    if ((int)dtype < 0 || (int)dtype > 3) return fail(SAM_ERR_UNSUPPORTED, "unknown dtype");
+    if ((int)dtype < 0 || (int)dtype > 5) return fail(SAM_ERR_UNSUPPORTED, "unknown dtype");
     if (order < 1 || order > 8) return fail(SAM_ERR_UNSUPPORTED, "order must be in 1..8 (DESIGN.md R4)");
     if (tuple < 1 || tuple > 8) return fail(SAM_ERR_UNSUPPORTED, "tuple must be in 1..8 (DESIGN.md R4)");
     return SAM_OK;
@@ -160,7 +165,7 @@ size_t pend_area(sam_dtype d, int k, int dev) {
 }
 
 int items_of(sam_dtype d) {
-    switch (d) {
+    switch (add_dtype(d)) {
         case SAM_I32: return sam::Cfg<uint32_t>::ITEMS;
         case SAM_I64: return sam::Cfg<uint64_t>::ITEMS;
         case SAM_F32: return sam::Cfg<float>::ITEMS;
@@ -240,7 +245,7 @@ int run_scan(sam_dtype dtype, int k, int s, int inclusive, const void* in, void*
     a.dev = dev;
     a.trace = g_trace;
     cudaError_t e;
-    switch (dtype) {
+    switch (add_dtype(dtype)) {
         case SAM_I32: e = dispatch_k<uint32_t>(k, a); break;
         case SAM_I64: e = dispatch_k<uint64_t>(k, a); break;
         case SAM_F32: e = dispatch_k<float>(k, a); break;
@@ -590,6 +595,54 @@ int sam_delta_encode_halo(sam_dtype dtype, int order, int tuple, const void* in,
     g_launches += l;
     return e == cudaSuccess ? SAM_OK : cuda_fail(e, "delta encoder launch");
 }
+
+int sam_scan_generic(sam_dtype dtype, sam_op op, sam_carry carry, int order, int tuple, int inclusive,
+                     const void* in, void* out, uint64_t n, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if ((int)op < 0 || (int)op > 3) return fail(SAM_ERR_UNSUPPORTED, "unknown operator");
+    if ((int)carry < 0 || (int)carry > 2) return fail(SAM_ERR_UNSUPPORTED, "unknown carry scheme");
+    if (op == SAM_OP_XOR && (dtype == SAM_F32 || dtype == SAM_F64))
+        return fail(SAM_ERR_UNSUPPORTED, "xor is defined for integer dtypes only (reading R14)");
+    rc = validate_buffers(dtype, in, out, n, true);
+    if (rc) return rc;
+    if (n == 0) return SAM_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* ws = nullptr;
+    int dev = 0;
+    rc = get_ws(st, sam::gen::generic_words_bytes((int)dtype, order, tuple, n), &ws, &dev);
+    if (rc) return rc;
+    sam::gen::GenArgs a;
+    memset(&a, 0, sizeof(a));
+    a.in = in;
+    a.out = out;
+    a.n = n;
+    a.s = tuple;
+    a.k = order;
+    a.inclusive = inclusive ? 1 : 0;
+    a.mode = (int)carry;
+    a.words = ws->carry;
+    a.words_bytes = ws->carry_cap;
+    a.tile_ctr = (unsigned long long*)(ws->ctr);
+    a.done_ctr = (unsigned int*)(ws->ctr + 8);
+    a.epoch_ptr = (unsigned int*)(ws->ctr + 12);
+    a.dev = dev;
+    a.num_sms = num_sms_of(dev);
+    a.stream = st;
+    a.mode_used = &g_last_carry;
+    cudaError_t e = sam::gen::launch_generic((int)dtype, (int)op, a);
+    if (e != cudaSuccess) return cuda_fail(e, "generic scan kernel launch");
+    g_launches += 1;
+    return SAM_OK;
+}
+
+int sam_scan_op(sam_dtype dtype, sam_op op, int order, int tuple, int inclusive, const void* in, void* out,
+                uint64_t n, sam_stream_t stream) {
+    if (op == SAM_OP_ADD) return sam_scan(dtype, order, tuple, inclusive, in, out, n, stream);
+    return sam_scan_generic(dtype, op, SAM_CARRY_STATIC, order, tuple, inclusive, in, out, n, stream);
+}
+
+int sam_last_carry_scheme(void) { return g_last_carry; }
 
 int sam_debug_limit_grid(uint64_t max_ctas) {
     sam::debug_grid_limit() = max_ctas;

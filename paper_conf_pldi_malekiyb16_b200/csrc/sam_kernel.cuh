@@ -247,6 +247,8 @@ struct Params {
     T bn[K][32];          // b_d(-(v+1)*ITEMS), v < Pw    ([d][v]; integer similarity transform)
     T bq[8][K];           // b_d(q*Uw),     q < c
     T bqn[8][K];          // b_d(-q*Uw),    q < c         (integer similarity transform)
+    T bposP[K];           // b_d(P*M*U)     (global-frame carries: one round further)
+    T bnegP[K];           // b_d(-P*M*U)
     CT bl[32][K];         // b_d(j*M*U),    j < Wn
     CT bsub[8][K];        // b_d(j*U),      j < M         (sub-tile offsets in a super-tile)
     T bks[5][K];          // b_d(2^l*ITEMS) (Kogge-Stone warp scan of thread states, K >= 3)
@@ -719,6 +721,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // published for the other CTAs' look-backs (a4).
         const int npair = s * c;
         T Pref[2][K];
+        T gneg[K];  // global frame (integers): b(-(S+1) US) of this CTA's current super-tile
+        if constexpr (TRANSFORM) mcol<T>(-((int64_t)blockIdx.x + 1) * p.M * p.U, K, gneg);
         for (int i = 0;; ++i) {
             const int qs = i % NQ;
             if (!wait_or_end(&bar_p1[qs], (uint32_t)((i / NQ) & 1), i)) break;
@@ -849,11 +853,21 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
                         }
                         if (jsub == cnt - 1) {
+                            T av[K];
+#pragma unroll
+                            for (int t = 0; t < K; ++t) av[t] = Pref[ch][t];
+                            if constexpr (TRANSFORM) {  // global frame: A~_S = M(-(S+1) US) A_S
+#pragma unroll
+                                for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                                    for (int j = 0; j < t; ++j) av[t] += gneg[t - j] * av[j];
+                                }
+                            }
 #pragma unroll
                             for (int t = 0; t < K; ++t) {
-                                la[mm * K + t] = Pref[ch][t];  // super-tile aggregate
+                                la[mm * K + t] = av[t];  // super-tile aggregate (transformed for integers)
                                 {  // a4: publish it
-                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W1, tag, Pref[ch][t]);
+                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W1, tag, av[t]);
                                 }
                             }
                         }
@@ -863,6 +877,18 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             __syncwarp();
             if (lane == 0) SAM_TRACE(3, tile);
             mbar_arrive(&bar_agg[qs]);
+            if (TRANSFORM && jsub == cnt - 1) {  // next super-tile of this CTA: one round further
+                T ng[K];
+#pragma unroll
+                for (int d = 0; d < K; ++d) {
+                    T acc2 = T(0);
+#pragma unroll
+                    for (int e2 = 0; e2 <= d; ++e2) acc2 += gneg[e2] * p.bnegP[d - e2];
+                    ng[d] = acc2;
+                }
+#pragma unroll
+                for (int d = 0; d < K; ++d) gneg[d] = ng[d];
+            }
             if (jsub == cnt - 1) {  // super-tile complete: wake its carry warp (super-tiles round-robin)
                 const int r = i / p.M;
                 // at most one unconsumed phase per barrier: the warp must have taken super-tile r-NCARRY
@@ -897,6 +923,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         const bool use_land = coop && S::LANDB > 0 &&
                               (uint64_t)(gridDim.x - 1) * s * SUPB + 32 <= (uint64_t)S::LANDB;
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
+        CT gpos[K];     // global frame: b(S US) of the current super-tile (lead, coop: advanced per round)
+        CT tsum[K];     // global frame: I~_prev + sum of the folded A~_j (the next hand-off adds A~_S)
+#pragma unroll
+        for (int t = 0; t < K; ++t) { gpos[t] = CT(0); tsum[t] = CT(0); }
         for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
             const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
@@ -1052,6 +1082,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         if (vv == V - 1) {
 #pragma unroll
                             for (int t = 0; t < K; ++t) Y[t] = X[t];
+                        } else if constexpr (TRANSFORM) {  // global frame: aggregates just add
+#pragma unroll
+                            for (int t = 0; t < K; ++t) Y[t] += X[t];
                         } else {
 #pragma unroll
                             for (int t = K - 1; t >= 0; --t) {  // Y <- M(Wn US) Y + X
@@ -1062,7 +1095,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             }
                         }
                     }
-                    if (active) {  // Y <- M(jl US) Y
+                    if (active && !TRANSFORM) {  // Y <- M(jl US) Y
 #pragma unroll
                         for (int t = K - 1; t >= 1; --t) {
                             CT acc2 = Y[t];
@@ -1079,6 +1112,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
                     }
                     // lanes jl == 0 hold this window's sum; total += M(j WV US) Y
+                    if constexpr (TRANSFORM) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) total[t] += Y[t];
+                    } else {
 #pragma unroll
                     for (int t = K - 1; t >= 0; --t) {
                         CT acc2 = Y[t];
@@ -1086,8 +1123,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int jj = 0; jj < t; ++jj) acc2 += Pm[t - jj] * Y[jj];
                         total[t] += acc2;
                     }
+                    }
                     if (last) break;
-                    {   // Pm <- Pm * M(jstep*WV*US)  (truncated polynomial product)
+                    if (!TRANSFORM) {   // Pm <- Pm * M(jstep*WV*US)  (truncated polynomial product)
                         CT np[K];
 #pragma unroll
                         for (int d = 0; d < K; ++d) {
@@ -1135,7 +1173,40 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         mcol<CT>(tile * (int64_t)p.M * p.U, K, bcol);
                         have = true;
                     }
-                    if (have) {
+                    if constexpr (TRANSFORM) {
+                        // global frame (integers): A~_j = M(-(j+1) US) A_j were published, so the fold
+                        // is a plain sum and the chain is a sum too: T~ = I~_prev + sum A~_j, and
+                        // C_S = M(S US) T~ (gpos = b(S US), advanced by one round per super-tile)
+                        if (have) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) total[t] += pv[t];
+                        }
+#pragma unroll
+                        for (int t = 0; t < K; ++t) tsum[t] = total[t];
+                        if (coop) {
+                            if (r == 0) {
+                                mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
+                            } else {
+                                CT np2[K];
+#pragma unroll
+                                for (int d = 0; d < K; ++d) {
+                                    CT acc2 = CT(0);
+#pragma unroll
+                                    for (int e2 = 0; e2 <= d; ++e2) acc2 += gpos[e2] * p.bposP[d - e2];
+                                    np2[d] = acc2;
+                                }
+#pragma unroll
+                                for (int d = 0; d < K; ++d) gpos[d] = np2[d];
+                            }
+                        } else {
+                            mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
+                        }
+#pragma unroll
+                        for (int t = K - 1; t >= 1; --t) {
+#pragma unroll
+                            for (int jj = 0; jj < t; ++jj) total[t] += gpos[t - jj] * total[jj];
+                        }
+                    } else if (have) {
 #pragma unroll
                         for (int t = K - 1; t >= 0; --t) {
                             CT acc2 = total[t] + pv[t];
@@ -1163,12 +1234,17 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 __syncwarp();
                 unsigned char* ho = smem + S::OFF_HO + (r % NCARRY) * S::HOB;
                 if (lane_ok) {
+                    if constexpr (TRANSFORM) {  // I~_S = T~ + A~_S (la holds the transformed aggregate)
+#pragma unroll
+                        for (int t = 0; t < K; ++t) ((CT*)(ho + 16))[lane * K + t] = tsum[t] + la[ml * K + t];
+                    } else {
 #pragma unroll
                     for (int t = 0; t < K; ++t) {
                         CT acc2 = C[t] + la[ml * K + t];
 #pragma unroll
                         for (int j = 0; j < t; ++j) acc2 += p.bus[t - j] * C[j];
                         ((CT*)(ho + 16))[lane * K + t] = acc2;
+                    }
                     }
                 }
                 __syncwarp();

@@ -240,6 +240,8 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
                 mcol<CT>(US, K, t->bus);
                 for (int j = 0; j <= NCARRY; ++j) mcol<CT>((int64_t)j * geo.Wn * Vr * US, K, t->bwinj[j]);
                 mcol<CT>((int64_t)(P - 1) * US, K, t->bprev);
+                mcol<T>((int64_t)P * US, K, t->bposP);
+                mcol<T>(-(int64_t)P * US, K, t->bnegP);
                 mcol<CT>((int64_t)geo.Wn * US, K, t->bwn);
                 for (int v = 0; v < 32; ++v) {
                     T b[K];
