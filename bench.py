@@ -196,6 +196,65 @@ def run_sweep(sam, synth, torch, peak, reps=5):
     return out
 
 
+def time_sharded(sam, synth, torch, dist, dt, n_local, k, s, rank, world, local, reps=5):
+    """One sharded step (sam_shard_state -> NCCL all-gather of the payloads -> sam_shard_scan) on
+    n_local elements per rank, CUDA events on the launching stream, max over ranks; plus the state
+    pass alone (its cost relative to the scan: the reduce-then-scan overhead)."""
+    import ctypes
+
+    free, _ = torch.cuda.mem_get_info()
+    w = W_BYTES[dt]
+    if free < 2 * n_local * w + (3 << 30):
+        return {"skipped": f"needs {2 * n_local * w / 2**30:.0f} GiB free HBM per GPU"}
+    g_off = rank * n_local
+    x = synth.make_torch(n_local, dt, "uniform", seed=synth.SEED_BASE + 5, start=g_off, device=torch.device("cuda", local))
+    y = torch.empty_like(x)
+    dc = sam.dtype_code(x.dtype)
+    st = torch.cuda.current_stream()
+    sp = ctypes.c_void_p(st.cuda_stream)
+    P = lambda t: ctypes.c_void_p(t.data_ptr())
+    pb = sam.sam_shard_payload_bytes(dc, k, s)
+    payload = torch.empty(pb, dtype=torch.uint8, device=x.device)
+    gathered = torch.empty(world * pb, dtype=torch.uint8, device=x.device)
+
+    def state():
+        sam.sam_shard_state(dc, k, s, P(x), n_local, g_off, P(payload), sp)
+
+    def step():
+        state()
+        if world > 1:
+            dist.all_gather_into_tensor(gathered, payload)
+        else:
+            gathered.copy_(payload)
+        sam.sam_shard_scan(dc, k, s, True, P(x), P(y), n_local, g_off, P(gathered), rank, world, sp)
+
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    res = {}
+    for name, fn in (("step", step), ("state", state)):
+        for _ in range(2):
+            fn()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        e0.record(st)
+        for _ in range(reps):
+            fn()
+        e1.record(st)
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1) / reps], dtype=torch.float64, device=x.device)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        res[name + "_ms"] = float(t[0])
+    n_total = n_local * world
+    res.update({"n_per_gpu": n_local, "n_total": n_total, "order": k, "tuple": s, "dtype": DTYPE_NAME[dt],
+                "gvalues_s": n_total / (res["step_ms"] * 1e-3) / 1e9,
+                "per_gpu_hbm_gbs_algorithmic": 2 * w * n_local / (res["step_ms"] * 1e-3) / 1e9,
+                "state_over_step": res["state_ms"] / res["step_ms"]})
+    del x, y
+    torch.cuda.empty_cache()
+    return res
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -473,10 +532,17 @@ def main():
 
     peak, peak_src = measured_peaks()
     sweep = None
-    if world == 1 and not args.no_sweep and not delta:
+    sharded = None
+    if not args.no_sweep and not delta:
         del y
         torch.cuda.empty_cache()
-        sweep = run_sweep(sam, synth, torch, peak)
+        if world == 1:
+            sweep = run_sweep(sam, synth, torch, peak)
+        # north_star's multi-GPU config C5 (int64, order 4, tuple 4): weak (2^30 per GPU) and strong
+        # (2^33 in total) through the sharded path, max over ranks; and the state pass alone (K*2)
+        sharded = {}
+        for tag, nl in (("c5_weak", 1 << 30), ("c5_strong", (1 << 33) // world)):
+            sharded[tag] = time_sharded(sam, synth, torch, dist, "i64", nl, 4, 4, rank, world, local)
     alg_bytes = 2 * w * n_local
     achieved = alg_bytes / (kavg * 1e-3) / 1e9
     if rank == 0:
@@ -498,6 +564,7 @@ def main():
                          "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
             "cpu_baseline": cpu,
             "sweep": sweep,
+            "sharded_c5": sharded,
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk.summary(),

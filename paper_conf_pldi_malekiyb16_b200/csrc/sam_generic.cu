@@ -25,8 +25,10 @@ cudaError_t launch_t(const GenArgs& a) {
     {
         std::lock_guard<std::mutex> lk(mu);
         if (!attr_set[a.dev]) {
+            size_t mx = 0;
+            for (int ss = 1; ss <= 8; ++ss) mx = S::bytes(ss) > mx ? S::bytes(ss) : mx;
             cudaError_t e = cudaFuncSetAttribute(sam_generic_kernel<T, OP, K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                 (int)S::bytes(8));
+                                                 (int)mx);
             if (e != cudaSuccess) return e;
             attr_set[a.dev] = true;
         }
@@ -42,7 +44,7 @@ cudaError_t launch_t(const GenArgs& a) {
     p.in = (const T*)a.in;
     p.out = (T*)a.out;
     p.n = a.n;
-    const uint64_t TT = (uint64_t)TB * S::IPS * a.s;
+    const uint64_t TT = (uint64_t)TB * Ips<T>::of(a.s) * a.s;
     p.num_tiles = (a.n + TT - 1) / TT;
     p.s = a.s;
     p.k = a.k;
@@ -142,7 +144,7 @@ cudaError_t launch_generic(int elem, int op, const GenArgs& a) {
 // workspace bytes of tagged words for n elements
 size_t generic_words_bytes(int elem, int k, int s, uint64_t n) {
     const int w = (elem == 0 || elem == 2 || elem == 4) ? 4 : 8;
-    const uint64_t TT = (uint64_t)TB * (w == 4 ? 4 : 2) * s;
+    const uint64_t TT = (uint64_t)TB * (w == 4 ? Ips<uint32_t>::of(s) : Ips<uint64_t>::of(s)) * s;
     const uint64_t tiles = (n + TT - 1) / TT + 1;
     return (size_t)tiles * s * 8 /* K <= 8 */ * 2 * (w / 4) * 8;
     (void)k;

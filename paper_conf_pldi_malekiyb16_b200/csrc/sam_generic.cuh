@@ -46,8 +46,11 @@ enum { GEN_STATIC = 0, GEN_LOOKBACK = 1, GEN_CHAINED = 2 };
 constexpr int TB = 256;    // threads per CTA
 constexpr int NWG = TB / 32;
 
-// lane positions per lane per thread: a tile is TB * IPS * s elements, IPS * TB positions per lane
-template <typename T> struct Ips { static constexpr int V = sizeof(T) == 4 ? 4 : 2; };
+// lane positions per lane per thread: a tile is TB * ips(s) * s elements (~16 KB for any s)
+template <typename T> struct Ips {
+    static constexpr int BASE = sizeof(T) == 4 ? 16 : 8;
+    static __host__ __device__ constexpr int of(int s) { return BASE / s > 1 ? BASE / s : 1; }
+};
 
 template <typename T, int OP> struct Op;
 template <typename T> struct Op<T, OP_ADD> {
@@ -146,10 +149,9 @@ __device__ __forceinline__ int pad(int e) { return e + (e >> 5); }  // one pad w
 
 template <typename T, int OP, int K>
 struct GSmem {
-    static constexpr int IPS = Ips<T>::V;
     // dynamic shared memory of a launch with tuple size s: two padded tiles + warp totals + states
     static constexpr size_t bytes(int s) {
-        const int TT = TB * IPS * s;
+        const int TT = TB * Ips<T>::of(s) * s;
         return (size_t)(2 * (TT + TT / 32 + 8) + NWG * 8 + 3 * 8 * K) * sizeof(T);
     }
 };
@@ -235,7 +237,8 @@ sam_generic_kernel(const __grid_constant__ GParams<T, K> p) {
     constexpr int W1 = GW<T>::W;
     extern __shared__ __align__(16) unsigned char smem[];
     const int s = p.s;
-    const int U = TB * S::IPS;               // lane positions per tile
+    const int IPS = Ips<T>::of(s);
+    const int U = TB * IPS;                  // lane positions per tile
     const int TT = U * s;                    // tile elements
     const int BUF = TT + TT / 32 + 8;        // padded buffer
     T* xs = (T*)smem;
@@ -247,7 +250,7 @@ sam_generic_kernel(const __grid_constant__ GParams<T, K> p) {
     __shared__ long long sh_tile;
     __shared__ unsigned sh_tag;
     const int tid = threadIdx.x, lane = tid & 31;
-    const int items = S::IPS * s;
+    const int items = IPS * s;
     const int kk = LIN ? K : p.k;             // state length (idempotent ops: the shift k)
     if (tid == 0) sh_tag = *(volatile unsigned*)p.epoch_ptr + 1u;
     __syncthreads();

@@ -128,6 +128,10 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_TRANSFORM
 #define SAM_TRANSFORM 1
 #endif
+// carry folds read their aggregates through one bulk copy into a smem landing buffer
+#ifndef SAM_LAND
+#define SAM_LAND 1
+#endif
 #ifndef SAM_KS_MIN_K
 #define SAM_KS_MIN_K 3
 #endif
@@ -466,7 +470,8 @@ struct SmemL {
     static constexpr int HOB = 16 + MAXS * K * (int)sizeof(CT);          // hand-off entry: i32 r, pad, [MAXS][K]
     static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
     static constexpr int OFF_PART = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;   // [2][NCARRY][MAXS][K]
-    static constexpr int OFF_EQ = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(CT);  // [ELAG][TILE_THREADS][K]
+    static constexpr int OFF_PV = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(CT);  // [NCARRY][64] value-parallel fold partials
+    static constexpr int OFF_EQ = OFF_PV + NCARRY * 64 * (int)sizeof(CT);                // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES0 = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
     // carry-fold landing buffer: the P-1 aggregates a fold reads, pulled from L2 in ONE bulk copy
     // (whatever shared memory is left, up to 40 KB; the fold falls back to windowed loads if short)
@@ -668,8 +673,21 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     else if (later == 1) bulk_wait_read<1>();
                     else if (later == 2) bulk_wait_read<2>();
                     else bulk_wait_read<3>();
-                    load_tile(tile_of[j2 % NQ], smem + S::OFF_BUF2 + (j2 % NB2) * S::BUFB, &bar_full2[j2 % NB2],
-                              pol_stream);
+                    // state-only pass (sam_shard_state): a tile holding no lane's last element needs
+                    // no carry application, so it is not re-fetched -- the barrier is just released
+                    bool need = true;
+                    if (p.store_mode == STORE_NONE) {
+                        const int64_t t0 = tile_of[j2 % NQ] * (int64_t)Tt;
+                        need = false;
+                        for (int mm = 0; mm < s; ++mm)
+                            need |= (p.last_e[mm] >= t0 && p.last_e[mm] < t0 + Tt);
+                    }
+                    if (need) {
+                        load_tile(tile_of[j2 % NQ], smem + S::OFF_BUF2 + (j2 % NB2) * S::BUFB, &bar_full2[j2 % NB2],
+                                  pol_stream);
+                    } else {
+                        mbar_arrive(&bar_full2[j2 % NB2]);
+                    }
                     ++j2;
                     continue;
                 }
@@ -920,7 +938,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // arrives in shared memory with one bulk copy; words whose tag is not yet this launch's are
         // re-polled from L2 (the nearest predecessors, published last)
         constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
-        const bool use_land = coop && S::LANDB > 0 &&
+        const bool use_land = SAM_LAND && coop && S::LANDB > 0 &&
                               (uint64_t)(gridDim.x - 1) * s * SUPB + 32 <= (uint64_t)S::LANDB;
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
         CT gpos[K];     // global frame: b(S US) of the current super-tile (lead, coop: advanced per round)
@@ -994,7 +1012,85 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                 for (int t = 0; t < K; ++t) { total[t] = CT(0); Pm[t] = p.bwinj[j0][t]; }  // Pm = M(j0 WV US)
                 int npoll = 0;
-                for (int j = j0;; j += jstep) {
+                // Integers with the landing buffer: the global-frame fold is a plain sum of the
+                // transformed aggregates, done value-parallel -- lane <-> (super-tile stripe, value
+                // (m, t)), consecutive lanes on consecutive words (conflict-free smem reads), the 4
+                // carry warps on interleaved super-tiles; stale words are re-polled from L2 one by one.
+                const bool vfold = TRANSFORM && land_r;
+                if (vfold) {
+                    // lane <-> (stripe st, value vi) for s*K <= 32 (stripes of super-tiles side by side),
+                    // lane <-> (vi, vi + 32) otherwise; warp cw takes stripes cw*ST + st, + NCARRY*ST, ...
+                    const int VPT = s * K;
+                    const int VL = VPT > 32 ? 32 : VPT;
+                    const int ST = 32 / VL;             // stripes per warp
+                    const int st = lane / VL, vi0 = lane - st * VL;
+                    const bool lact = st < ST;
+                    const int64_t nsup = tile - lo_sup;
+                    CT acc[2][2] = {{CT(0), CT(0)}, {CT(0), CT(0)}};  // [h][parity]: two chains for ILP
+                    if (p.trace && lead && lane == 0) SAM_TRACE(8, tile * p.M);
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int vi = vi0 + 32 * h;
+                        if (!lact || vi >= VPT) continue;
+                        int par = 0;
+                        for (int64_t jj = (int64_t)cw * ST + st; jj < nsup; jj += (int64_t)NCARRY * ST, par ^= 1) {
+                            const unsigned long long* src = p.carry + ((size_t)(lo_sup + jj) * VPT + vi) * W1;
+                            const unsigned long long* ls =
+                                (const unsigned long long*)(smem + S::OFF_LAND + ((uintptr_t)src - land_a16));
+                            unsigned long long w0 = ls[0], w1 = W1 == 2 ? ls[1] : 0ull;
+                            while ((uint32_t)(w0 >> 32) != tag || (W1 == 2 && (uint32_t)(w1 >> 32) != tag)) {
+                                if constexpr (W1 == 1) {
+                                    w0 = ld_relaxed_u64(src);
+                                } else {
+                                    ld_relaxed_v2(src, w0, w1);
+                                }
+                                ++npoll;
+                            }
+                            const uint64_t b = W1 == 1 ? (w0 & 0xffffffffull) : ((w0 & 0xffffffffull) | (w1 << 32));
+                            acc[h][par] += CT(Bits<T>::from(b));
+                        }
+                    }
+                    CT v0 = acc[0][0] + acc[0][1], v1 = acc[1][0] + acc[1][1];
+                    // stripes -> stripe 0 (tree over st; ST need not be a power of two)
+                    for (int step = 1; step < ST; step <<= 1) {
+                        const CT o = shfl_down(v0, step * VL);
+                        if (lact && (st % (2 * step)) == 0 && st + step < ST) v0 += o;
+                    }
+                    CT* pv_s = (CT*)(smem + S::OFF_PV);  // [NCARRY][64]
+                    if (st == 0) {
+                        pv_s[cw * 64 + vi0] = v0;
+                        pv_s[cw * 64 + 32 + vi0] = v1;
+                    }
+                    named_bar_sync(4, NCARRY * 32);
+                    if (lead) {
+                        // value vi summed over the warps by lane vi, then lane m collects its K values
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int vi = lane + 32 * h;
+                            if (vi < VPT) {
+                                const int slot = vi < 32 ? vi : 32 + (vi - 32);
+                                CT a2 = pv_s[slot];
+#pragma unroll
+                                for (int w2 = 1; w2 < NCARRY; ++w2) a2 += pv_s[w2 * 64 + slot];
+                                pv_s[slot] = a2;
+                            }
+                        }
+                        __syncwarp();
+                        if (lane_ok) {
+#pragma unroll
+                            for (int t = 0; t < K; ++t) {
+                                const int vi = lane * K + t;
+                                total[t] = pv_s[vi < 32 ? vi : 32 + (vi - 32)];
+                            }
+                        }
+                        if (lane == 0) {
+                            SAM_TRACE(10, tile * p.M);
+                            SAM_TRACE(13, tile * p.M);
+                            if (p.trace) p.trace[(size_t)(tile * p.M) * 16 + 11] = npoll;
+                        }
+                    }
+                }
+                for (int j = j0; !vfold; j += jstep) {
                     const int64_t basei = tile - 1 - (int64_t)j * WV;
                     if (basei < Sprev) break;  // window j starts beyond Sprev: nothing left for this warp
                     unsigned long long w[V][K][W1];
@@ -1138,7 +1234,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int d = 0; d < K; ++d) Pm[d] = np[d];
                     }
                 }
-                if (coop) {  // sum the warps' partial folds (all already at their absolute offsets)
+                if (coop && !vfold) {  // sum the warps' partial folds (all already at their absolute offsets)
                     CT* slot = part_s + ((r & 1) * NCARRY + cw) * MAXS * K;
                     if (lane_ok) {
 #pragma unroll
