@@ -132,11 +132,21 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_LAND
 #define SAM_LAND 1
 #endif
+#ifndef SAM_TR32_MIN_K
+#define SAM_TR32_MIN_K 2
+#endif
 #ifndef SAM_KS_MIN_K
 #define SAM_KS_MIN_K 3
 #endif
 #ifndef SAM_LAG8
 #define SAM_LAG8 12
+#endif
+#ifndef SAM_LAG16
+#define SAM_LAG16 8
+#endif
+// max tiles per super-tile for states > 8 B (the carry team's work is per super-tile)
+#ifndef SAM_MMAX_BIG
+#define SAM_MMAX_BIG 2
 #endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
@@ -169,9 +179,9 @@ template <typename T, int K> struct Lag {
     // bounded by shared memory
     static constexpr bool GPEND = SAM_GPEND && SB > 16;
     static constexpr bool SMEM = !GPEND && (SB <= 16 || BIG32 || BIG64);  // pending local states in shared memory
-    static constexpr int LAG = GPEND ? SAM_LAGG : (SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? 8 : (BIG32 ? SAM_LAG32 : SAM_LAG64))));
+    static constexpr int LAG = GPEND ? SAM_LAGG : (SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? SAM_LAG16 : (BIG32 ? SAM_LAG32 : SAM_LAG64))));
     // max tiles per super-tile (look-back unit); measured: 3 for 4-byte, 2 for 8-byte elements
-    static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : 2;
+    static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : (SB <= 8 ? 2 : SAM_MMAX_BIG);
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
     static constexpr int NB2 = SB <= 8 ? 4 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
@@ -230,6 +240,8 @@ struct Params {
     int64_t last_e[MAXS]; // virtual index of lane m's last element, -1 if none
     T* pend;              // GPEND: pending local states [grid][LAG][K][TILE_THREADS] (workspace)
     int lag;              // pipeline depth used (1..LAG): max tiles between a local scan and its carry application
+    int land;             // carry folds read through the smem landing buffer (when it fits)
+    int vfold;            // integers + landing: value-parallel fold (else the windowed fold from the buffer)
     unsigned long long* carry;  // tagged carry words: [tile][m][t][agg W | incl W]
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
@@ -514,7 +526,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     constexpr int PF = S::NB1;  // max claimed-but-unscanned tiles
     constexpr int W1 = TagW<T>::W;      // tagged words per published value
     constexpr int V = LB<T, K>::V;
-    constexpr bool TRANSFORM = IsInt<T>::value && K >= 2 && SAM_TRANSFORM;  // integer similarity-transform scans
+    // integer similarity-transform scans / global-frame carries (int32: from order SAM_TR32_MIN_K)
+    constexpr bool TRANSFORM = IsInt<T>::value && K >= 2 && SAM_TRANSFORM && (sizeof(T) == 8 || K >= SAM_TR32_MIN_K);
     static_assert(ITEMS >= K, "exclusive shift needs ITEMS >= K");
     static_assert(VEC || ITEMS % 2 == 1, "ITEMS odd keeps the stride-s smem reads bank-conflict free");
     static_assert(PF <= NB1 && NQ > LAG && NQ > NB1 && NB2 <= 4, "ring sizes");
@@ -938,7 +951,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // arrives in shared memory with one bulk copy; words whose tag is not yet this launch's are
         // re-polled from L2 (the nearest predecessors, published last)
         constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
-        const bool use_land = SAM_LAND && coop && S::LANDB > 0 &&
+        const bool use_land = SAM_LAND && p.land && coop && S::LANDB > 0 &&
                               (uint64_t)(gridDim.x - 1) * s * SUPB + 32 <= (uint64_t)S::LANDB;
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
         CT gpos[K];     // global frame: b(S US) of the current super-tile (lead, coop: advanced per round)
@@ -1016,7 +1029,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 // transformed aggregates, done value-parallel -- lane <-> (super-tile stripe, value
                 // (m, t)), consecutive lanes on consecutive words (conflict-free smem reads), the 4
                 // carry warps on interleaved super-tiles; stale words are re-polled from L2 one by one.
-                const bool vfold = TRANSFORM && land_r;
+                const bool vfold = TRANSFORM && land_r && p.vfold;
                 if (vfold) {
                     // lane <-> (stripe st, value vi) for s*K <= 32 (stripes of super-tiles side by side),
                     // lane <-> (vi, vi + 32) otherwise; warp cw takes stripes cw*ST + st, + NCARRY*ST, ...

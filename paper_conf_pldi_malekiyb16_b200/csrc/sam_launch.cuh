@@ -82,6 +82,8 @@ struct Knobs {
     int coop = -1;         // SAM_COOP: carry warps fold each super-tile together (1) or round-robin (0)
     bool no_vec = false;   // SAM_NO_VEC: never take the 128-bit tuple-1 path
     int lag = 0;           // SAM_LAG: pipeline depth (tiles between local scan and carry application), <= LAG
+    int land = -1;         // SAM_LAND: landing-buffer folds on (1) / off (0)
+    int vfold = -1;        // SAM_VFOLD: value-parallel integer folds on (1) / off (0)
 };
 inline const Knobs& knobs() {
     static const Knobs k = [] {
@@ -92,6 +94,8 @@ inline const Knobs& knobs() {
         if (const char* e = getenv("SAM_COOP")) r.coop = atoi(e) != 0;
         r.no_vec = getenv("SAM_NO_VEC") != nullptr;
         if (const char* e = getenv("SAM_LAG")) r.lag = atoi(e);
+        if (const char* e = getenv("SAM_LAND")) r.land = atoi(e) != 0;
+        if (const char* e = getenv("SAM_VFOLD")) r.vfold = atoi(e) != 0;
         return r;
     }();
     return k;
@@ -289,6 +293,10 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         p.reset_ctr = a.reset_ctr;
         p.pend = (T*)a.pend;
         p.lag = (kn.lag >= 1 && kn.lag <= S::LAG) ? kn.lag : S::LAG;
+        p.land = kn.land >= 0 ? kn.land : 1;
+        // measured (profiles/r2_ab_matrix.txt): the value-parallel fold wins from s*k >= 4 values per
+        // super-tile (int64 k=4: +3%, C5: +16%), the windowed fold below (int64 k=2/3: +4-7%)
+        p.vfold = kn.vfold >= 0 ? kn.vfold : (a.s * K >= 4 ? 1 : 0);
         p.trace = a.trace;
         p.stress = debug_stress();
 
