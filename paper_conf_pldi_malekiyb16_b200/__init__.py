@@ -16,7 +16,7 @@ import os
 __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
     "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_scan_workspace_size", "sam_scan_ws",
-    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_scan_op", "sam_scan_generic", "sam_last_carry_scheme",
+    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_scan_op", "sam_scan_generic", "sam_last_carry_scheme", "sam_tune_override",
     "scan_op", "SAM_U32", "SAM_U64", "SAM_OP", "SAM_CARRY", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
     "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "sam_delta_encode_host", "delta_encode_host", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
@@ -69,6 +69,7 @@ def lib() -> ctypes.CDLL:
             "sam_scan_op": (I, [I, I, I, I, I, P, P, U64, P]),
             "sam_scan_generic": (I, [I, I, I, I, I, I, P, P, U64, P]),
             "sam_last_carry_scheme": (I, []),
+            "sam_tune_override": (I, [I, I, I, I]),
             "sam_debug_set_stress": (I, [ctypes.c_uint32]),
             "sam_scan_workspace_size": (I, [I, I, I, U64, ctypes.POINTER(SZ)]),
             "sam_scan_ws": (I, [I, I, I, I, P, P, U64, P, SZ, P]),
@@ -121,6 +122,10 @@ def sam_scan_op(dtype, op, order, tuple_, inclusive, in_ptr, out_ptr, n, stream=
 def sam_scan_generic(dtype, op, carry, order, tuple_, inclusive, in_ptr, out_ptr, n, stream=None) -> int:
     return _check(lib().sam_scan_generic(dtype, op, carry, order, tuple_, int(bool(inclusive)), in_ptr, out_ptr, n,
                                          stream))
+
+
+def sam_tune_override(tiles_per_unit=-1, lag=-1, vfold=-1, land=-1) -> int:
+    return _check(lib().sam_tune_override(tiles_per_unit, lag, vfold, land))
 
 
 def sam_last_carry_scheme() -> int:

@@ -173,10 +173,19 @@ int items_of(sam_dtype d) {
     }
 }
 
-// bytes of tagged carry words for `tiles` tiles (an upper bound of the super-tiles): per (super-tile,
-// lane, order) one value in 1 (4-byte types) or 2 (8-byte types) 64-bit words
+// bytes of the O(1) carry ring (sam_launch.cuh): RING_ROUNDS records per CTA of the largest grid of
+// the current device, whatever n is (`tiles` is no longer needed)
 size_t carry_bytes(sam_dtype d, int k, int s, size_t tiles) {
-    return tiles * (size_t)s * (size_t)k * (elem_size(d) / 4) * 8;
+    (void)tiles;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    return sam::ring_bytes((int)elem_size(d), k, s, num_sms_of(dev));
+}
+// the largest ring of any (dtype, order, tuple): the generic kernel's words go after it
+size_t ring_max_bytes() {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    return sam::ring_bytes(8, 8, 8, num_sms_of(dev));
 }
 size_t tiles_for(sam_dtype dtype, int s, uint64_t n) {
     const sam::Geom geo = sam::make_geom(s, items_of(dtype));
@@ -610,7 +619,8 @@ int sam_scan_generic(sam_dtype dtype, sam_op op, sam_carry carry, int order, int
     cudaStream_t st = (cudaStream_t)stream;
     Workspace* ws = nullptr;
     int dev = 0;
-    rc = get_ws(st, sam::gen::generic_words_bytes((int)dtype, order, tuple, n), &ws, &dev);
+    const size_t rmax = ring_max_bytes();
+    rc = get_ws(st, rmax + sam::gen::generic_words_bytes((int)dtype, order, tuple, n), &ws, &dev);
     if (rc) return rc;
     sam::gen::GenArgs a;
     memset(&a, 0, sizeof(a));
@@ -621,8 +631,8 @@ int sam_scan_generic(sam_dtype dtype, sam_op op, sam_carry carry, int order, int
     a.k = order;
     a.inclusive = inclusive ? 1 : 0;
     a.mode = (int)carry;
-    a.words = ws->carry;
-    a.words_bytes = ws->carry_cap;
+    a.words = ws->carry + rmax / 8;  // after the main kernel's ring: separate tags and layout
+    a.words_bytes = ws->carry_cap - rmax;
     a.tile_ctr = (unsigned long long*)(ws->ctr);
     a.done_ctr = (unsigned int*)(ws->ctr + 8);
     a.epoch_ptr = (unsigned int*)(ws->ctr + 12);
@@ -647,6 +657,15 @@ int sam_last_carry_scheme(void) { return g_last_carry; }
 int sam_debug_limit_grid(uint64_t max_ctas) {
     sam::debug_grid_limit() = max_ctas;
     for (int d = 0; d < sam::MAX_DEVICES; ++d) sam::debug_grid_cap(d) = 0;
+    return SAM_OK;
+}
+
+int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land) {
+    sam::Knobs& k = sam::knobs_mut();
+    k.super_tile = (tiles_per_unit >= 1 && tiles_per_unit <= 8) ? tiles_per_unit : 0;
+    k.lag = lag >= 1 ? lag : 0;
+    k.vfold = vfold >= 0 ? (vfold != 0) : -1;
+    k.land = land >= 0 ? (land != 0) : -1;
     return SAM_OK;
 }
 

@@ -246,7 +246,9 @@ struct Params {
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
-    unsigned long long carry_words;  // capacity of `carry` (64-bit words)
+    unsigned long long carry_words;  // words of the carry ring actually used (R * rec_words)
+    unsigned long long ring;         // R: super-tile slots of the O(1) carry ring (a multiple of the grid)
+    unsigned int rec_words;          // words per super-tile record (16-B multiple)
     unsigned int* reset_ctr;         // grid barrier of the epoch wrap-around reset
     unsigned long long* trace;  // optional per-tile event timestamps [tile][8] (diagnostics), or null
     uint32_t stress;            // testing: nonzero = seed of pseudo-random delays at every pipeline hand-over
@@ -586,10 +588,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             *(volatile int*)(smem + S::OFF_HO + w * S::HOB) = -1;
         }
         fence_mbar_init();
-        // tags are never 0 (zero-filled workspace); when the 32-bit epoch wraps, this launch first
-        // zeroes every carry word (below) so no word tagged 2^32 launches ago can validate
+        // tag of a word = [20-bit launch epoch | 12-bit ring lap of its super-tile]; the epoch part
+        // cycles 1..2^20-1 (never 0: zero-filled memory never validates); when it restarts at 1 this
+        // launch first zeroes the ring (below) so no word of a launch 2^20-1 launches ago validates
         const unsigned ep = *(volatile unsigned int*)p.epoch_ptr;
-        *sm_tag = ep == 0xffffffffu ? 0u : ep + 1u;
+        const unsigned ep20 = ep % 1048575u + 1u;
+        *sm_tag = ep20 == 1u ? 0u : (ep20 << 12);
         *sm_end = -1;
         *agg_done = 0;
         *(volatile int*)(smem + S::OFF_TAG + 12) = 0;
@@ -600,7 +604,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     for (int i = tid; i < S::NBL * K; i += blockDim.x) bl_s[i] = (&p.bl[0][0])[i];
     for (int i = tid; i < 8 * K; i += blockDim.x) bq_s[i] = (&p.bq[0][0])[i];
     __syncthreads();
-    if (*sm_tag == 0u) {  // epoch wrap-around (once per 2^32 launches of a workspace)
+    if (*sm_tag == 0u) {  // epoch wrap-around (once per 2^20-1 launches of a workspace; the ring is small)
         for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + tid; i < p.carry_words;
              i += (unsigned long long)gridDim.x * blockDim.x)
             p.carry[i] = 0ull;
@@ -610,12 +614,17 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             atomicAdd(p.reset_ctr, 1u);
             while (*(volatile unsigned int*)p.reset_ctr < gridDim.x) __nanosleep(100);
             __threadfence();
-            *sm_tag = 1u;
-            if (blockIdx.x == 0) *(volatile unsigned int*)p.epoch_ptr = 0u;  // the epilogue makes it 1
+            *sm_tag = 1u << 12;
         }
         __syncthreads();
     }
-    const uint32_t tag = *sm_tag;
+    const uint32_t tag = *sm_tag;  // base tag: | ring lap of the super-tile
+    // O(1) carry ring: super-tile S lives in slot S mod R, tagged with its lap S / R, so a
+    // word of the previous lap (or launch) never validates
+    auto ctag = [&](int64_t S) -> uint32_t { return tag | (uint32_t)(((uint64_t)S / p.ring) & 0xfffu); };
+    auto cslot = [&](int64_t S) -> unsigned long long* {
+        return p.carry + ((uint64_t)S % p.ring) * p.rec_words;
+    };
 
     // wait for barrier phase `par`, or return false once the stream has ended before iteration it
     auto wait_or_end = [&](uint64_t* bar, uint32_t par, int it) -> bool {
@@ -898,7 +907,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                             for (int t = 0; t < K; ++t) {
                                 la[mm * K + t] = av[t];  // super-tile aggregate (transformed for integers)
                                 {  // a4: publish it
-                                    put_tagged<T>(p.carry + (((size_t)sup * s + mm) * K + t) * W1, tag, av[t]);
+                                    put_tagged<T>(cslot(sup) + (mm * K + t) * W1, ctag(sup), av[t]);
                                 }
                             }
                         }
@@ -952,7 +961,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // re-polled from L2 (the nearest predecessors, published last)
         constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
         const bool use_land = SAM_LAND && p.land && coop && S::LANDB > 0 &&
-                              (uint64_t)(gridDim.x - 1) * s * SUPB + 32 <= (uint64_t)S::LANDB;
+                              (uint64_t)(gridDim.x - 1) * p.rec_words * 8 <= (uint64_t)S::LANDB;
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
         CT gpos[K];     // global frame: b(S US) of the current super-tile (lead, coop: advanced per round)
         CT tsum[K];     // global frame: I~_prev + sum of the folded A~_j (the next hand-off adds A~_S)
@@ -971,13 +980,19 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             // the current round's (the nearest) are re-polled from L2 if not yet there.
             const int64_t lo_sup = Sprev + 1;
             const bool land_r = use_land && tile > lo_sup;
-            const uintptr_t land_a16 = ((uintptr_t)p.carry + (uintptr_t)lo_sup * s * SUPB) & ~(uintptr_t)15;
+            // landing offset of super-tile j: (j - lo_sup) * REC; the ring range may wrap: two copies
             if (land_r && lead && lane == 0) {
-                const uintptr_t b16 = ((uintptr_t)p.carry + (uintptr_t)tile * s * SUPB + 15) & ~(uintptr_t)15;
+                const uint64_t REC = (uint64_t)p.rec_words * 8;
+                const uint64_t cnt = (uint64_t)(tile - lo_sup);
+                const uint64_t slot0 = (uint64_t)lo_sup % p.ring;
+                const uint64_t c1 = slot0 + cnt <= p.ring ? cnt : p.ring - slot0;
                 fence_proxy_async_smem();  // the previous fold's generic reads of the buffer come first
-                mbar_arrive_expect_tx(bar_land, (uint32_t)(b16 - land_a16));
-                bulk_g2s(smem + S::OFF_LAND, (const void*)land_a16, (uint32_t)(b16 - land_a16), bar_land,
-                         policy_evict_last());
+                mbar_arrive_expect_tx(bar_land, (uint32_t)(cnt * REC));
+                bulk_g2s(smem + S::OFF_LAND, (const void*)(p.carry + slot0 * p.rec_words), (uint32_t)(c1 * REC),
+                         bar_land, policy_evict_last());
+                if (c1 < cnt)
+                    bulk_g2s(smem + S::OFF_LAND + c1 * REC, (const void*)p.carry, (uint32_t)((cnt - c1) * REC),
+                             bar_land, policy_evict_last());
             }
             if (lead) {
                 // Wait for the aggregator: it arrives on bar_cw[r % NCARRY] when super-tile r is
@@ -1047,11 +1062,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         if (!lact || vi >= VPT) continue;
                         int par = 0;
                         for (int64_t jj = (int64_t)cw * ST + st; jj < nsup; jj += (int64_t)NCARRY * ST, par ^= 1) {
-                            const unsigned long long* src = p.carry + ((size_t)(lo_sup + jj) * VPT + vi) * W1;
-                            const unsigned long long* ls =
-                                (const unsigned long long*)(smem + S::OFF_LAND + ((uintptr_t)src - land_a16));
+                            const unsigned long long* src = cslot(lo_sup + jj) + vi * W1;
+                            const unsigned long long* ls = (const unsigned long long*)(
+                                smem + S::OFF_LAND + ((size_t)jj * p.rec_words + vi * W1) * 8);
+                            const uint32_t tj = ctag(lo_sup + jj);
                             unsigned long long w0 = ls[0], w1 = W1 == 2 ? ls[1] : 0ull;
-                            while ((uint32_t)(w0 >> 32) != tag || (W1 == 2 && (uint32_t)(w1 >> 32) != tag)) {
+                            while ((uint32_t)(w0 >> 32) != tj || (W1 == 2 && (uint32_t)(w1 >> 32) != tj)) {
                                 if constexpr (W1 == 1) {
                                     w0 = ld_relaxed_u64(src);
                                 } else {
@@ -1122,10 +1138,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
                                 const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                                const unsigned long long* src = p.carry + ((size_t)idx * s + mlb) * K * W1;
+                                const unsigned long long* src = cslot(idx) + mlb * K * W1;
                                 if (from_land) {
                                     const unsigned long long* ls = (const unsigned long long*)(
-                                        smem + S::OFF_LAND + ((uintptr_t)src - land_a16));
+                                        smem + S::OFF_LAND + ((size_t)(idx - lo_sup) * p.rec_words + mlb * K * W1) * 8);
 #pragma unroll
                                     for (int t = 0; t < K; ++t) {
 #pragma unroll
@@ -1149,10 +1165,11 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
                                 bool ok = true;
+                                const uint32_t tv = ctag(basei - jl - (int64_t)Wn * vv);
 #pragma unroll
                                 for (int t = 0; t < K; ++t) {
-                                    ok &= (uint32_t)(w[vv][t][0] >> 32) == tag;
-                                    if constexpr (W1 == 2) ok &= (uint32_t)(w[vv][t][1] >> 32) == tag;
+                                    ok &= (uint32_t)(w[vv][t][0] >> 32) == tv;
+                                    if constexpr (W1 == 2) ok &= (uint32_t)(w[vv][t][1] >> 32) == tv;
                                 }
                                 st[vv] = ok ? 1 : 0;
                                 pend |= !ok;

@@ -6,8 +6,13 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include <dlfcn.h>
+#include <stdio.h>
+
 #include <map>
 #include <mutex>
+#include <string>
+#include <vector>
 
 #include "sam_algebra.h"
 #include "sam_kernel.cuh"
@@ -85,8 +90,8 @@ struct Knobs {
     int land = -1;         // SAM_LAND: landing-buffer folds on (1) / off (0)
     int vfold = -1;        // SAM_VFOLD: value-parallel integer folds on (1) / off (0)
 };
-inline const Knobs& knobs() {
-    static const Knobs k = [] {
+inline Knobs& knobs_mut() {
+    static Knobs k = [] {
         Knobs r;
         if (const char* e = getenv("SAM_CLAIM_SLACK")) { const int v = atoi(e); r.claim_slack = v < 0 ? 0 : (v > 2 ? 2 : v); }
         if (const char* e = getenv("SAM_SUPER_TILE")) { const int v = atoi(e); if (v >= 1 && v <= 8) r.super_tile = v; }
@@ -100,8 +105,63 @@ inline const Knobs& knobs() {
     }();
     return k;
 }
+inline const Knobs& knobs() { return knobs_mut(); }
 
 constexpr int MAX_DEVICES = 64;
+
+// Install-time autotune table (SAM's auto-tuner "runs when SAM is installed and determines the
+// optimal number of input elements to allocate to each thread for different ranges of problem
+// sizes").  Here the per-size-range choice is the carry unit -- tiles per super-tile M,
+// i.e. elements per CTA carry step -- and the pipeline depth, per (element type, order, tuple).
+// tools/autotune.py measures them on the installed GPU and writes lib/sam_tune.txt, one entry per line:
+//     <u32|u64|f32|f64> <k> <s> <log2 n lo> <log2 n hi> <M> <lag> <vfold> <land>
+// (M, lag: 0 = built-in default; vfold, land: 0 = default, 1 = off, 2 = on).  Loaded once; the
+// environment knobs still win.
+struct TuneEntry {
+    int w, isf, k, s, lo, hi, M, lag, vfold, land;
+};
+inline const std::vector<TuneEntry>& tune_table() {
+    static const std::vector<TuneEntry> t = [] {
+        std::vector<TuneEntry> r;
+        std::string path;
+        if (const char* e = getenv("SAM_TUNE_FILE")) {
+            path = e;
+        } else {
+            Dl_info di;
+            if (dladdr((void*)&tune_table, &di) && di.dli_fname) {
+                path = di.dli_fname;
+                const size_t slash = path.rfind('/');
+                path = (slash == std::string::npos ? std::string(".") : path.substr(0, slash)) + "/sam_tune.txt";
+            }
+        }
+        FILE* f = path.empty() ? nullptr : fopen(path.c_str(), "r");
+        if (!f) return r;
+        char line[256], ty[8];
+        while (fgets(line, sizeof(line), f)) {
+            TuneEntry e;
+            if (line[0] == '#') continue;
+            if (sscanf(line, "%7s %d %d %d %d %d %d %d %d", ty, &e.k, &e.s, &e.lo, &e.hi, &e.M, &e.lag, &e.vfold,
+                       &e.land) != 9)
+                continue;
+            e.w = (ty[1] == '6') ? 8 : 4;
+            e.isf = ty[0] == 'f';
+            r.push_back(e);
+        }
+        fclose(f);
+        return r;
+    }();
+    return t;
+}
+template <typename T>
+inline const TuneEntry* tune_lookup(int k, int s, uint64_t n) {
+    int lg = 0;
+    while (lg < 63 && (1ull << (lg + 1)) <= n) ++lg;
+    for (const TuneEntry& e : tune_table())
+        if (e.w == (int)sizeof(T) && e.isf == (int)std::is_floating_point<T>::value && e.k == k && e.s == s &&
+            lg >= e.lo && lg <= e.hi)
+            return &e;
+    return nullptr;
+}
 
 // Per-device launch facts of one kernel instantiation: the dynamic-shared-memory opt-in
 // (cudaFuncSetAttribute is per device context) and the occupancy, set on first use on each device.
@@ -155,6 +215,22 @@ inline uint32_t& debug_stress() {
     return seed;
 }
 
+// O(1) carry ring: R = RING_ROUNDS * grid super-tile records.  A slot is rewritten one
+// lap (RING_ROUNDS rounds) later by the same CTA; every reader of the old record is a fold of one of the
+// next P-1 super-tiles, and a CTA cannot run more than 2*LAG/M + 1 <= 25 rounds ahead of another's
+// carries (its local scans wait on its own carries, which wait on everyone's aggregates), so 32 rounds
+// leave margin; the lap in every word's tag turns a violation into a wait, never a wrong value.
+constexpr int RING_ROUNDS = 32;
+// 64-bit words per super-tile record: s*k values of 1 or 2 words, padded to 16 B (bulk copies)
+inline unsigned rec_words_of(int w, int k, int s) {
+    const unsigned words = (unsigned)(s * k * (w / 4));
+    return (words + 1u) & ~1u;
+}
+// bytes of the ring for a grid of `ctas`
+inline size_t ring_bytes(int w, int k, int s, int ctas) {
+    return (size_t)ctas * RING_ROUNDS * rec_words_of(w, k, s) * 8;
+}
+
 // global-memory pending-state scratch of one launch: [grid][LAG][K][TILE_THREADS] elements
 template <typename T, int K>
 constexpr size_t pend_bytes_tk(int num_ctas) {
@@ -193,6 +269,10 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
     }
     const Geom geo = make_geom(a.s, ITEMS);
     const uint64_t h = a.g % (uint64_t)a.s;
+    // pipeline depth: knob, else the autotune table, else the built-in LAG
+    const TuneEntry* te = tune_lookup<T>(K, a.s, a.n);
+    const int lag_rt = (kn.lag >= 1 && kn.lag <= S::LAG) ? kn.lag
+                       : ((te && te->lag >= 1 && te->lag <= S::LAG) ? te->lag : S::LAG);
     const uint64_t num_tiles = (h + a.n + geo.T - 1) / geo.T;
     // super-tile size: up to MMAX tiles per carry unit, but keep >= 2 super-tiles per SM
     uint64_t M;
@@ -203,10 +283,11 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         // 3, or 4 for odd tuples of 4-byte elements (~1.5% better there)
         const uint64_t mmax = a.s == 1 ? (uint64_t)Lag<T, K>::MMAX : ((sizeof(T) == 4 && (a.s & 1)) ? 4u : 3u);
         if (M > mmax) M = mmax;
+        if (te && te->M > 0) M = (uint64_t)te->M;
         if (kn.super_tile) M = (uint64_t)kn.super_tile;
         // a super-tile is aggregated before its carry is known: at most LAG/2 tiles per unit
         // keep two units in flight per CTA (LAG bounds the tiles between load and carry application)
-        const uint64_t mlag = Lag<T, K>::LAG / 2 > 1 ? Lag<T, K>::LAG / 2 : 1;
+        const uint64_t mlag = lag_rt / 2 > 1 ? (uint64_t)lag_rt / 2 : 1;
         if (M > mlag) M = mlag;
     }
     const uint64_t num_super = (num_tiles + M - 1) / M;
@@ -286,17 +367,21 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
             }
         }
         p.carry = a.carry;
-        p.carry_words = a.carry_words;
+        p.ring = P * RING_ROUNDS;
+        p.rec_words = rec_words_of((int)sizeof(T), K, a.s);
+        p.carry_words = p.ring * p.rec_words;
+        if (p.carry_words > a.carry_words) return cudaErrorInvalidValue;  // workspace too small for this grid
         p.tile_ctr = a.tile_ctr;
         p.done_ctr = a.done_ctr;
         p.epoch_ptr = a.epoch_ptr;
         p.reset_ctr = a.reset_ctr;
         p.pend = (T*)a.pend;
-        p.lag = (kn.lag >= 1 && kn.lag <= S::LAG) ? kn.lag : S::LAG;
-        p.land = kn.land >= 0 ? kn.land : 1;
+        const TuneEntry* tl = te;
+        p.lag = lag_rt;
+        p.land = kn.land >= 0 ? kn.land : ((tl && tl->land > 0) ? tl->land - 1 : 1);
         // measured (profiles/r2_ab_matrix.txt): the value-parallel fold wins from s*k >= 4 values per
         // super-tile (int64 k=4: +3%, C5: +16%), the windowed fold below (int64 k=2/3: +4-7%)
-        p.vfold = kn.vfold >= 0 ? kn.vfold : (a.s * K >= 4 ? 1 : 0);
+        p.vfold = kn.vfold >= 0 ? kn.vfold : ((tl && tl->vfold > 0) ? tl->vfold - 1 : (a.s * K >= 4 ? 1 : 0));
         p.trace = a.trace;
         p.stress = debug_stress();
 

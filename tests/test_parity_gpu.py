@@ -316,9 +316,10 @@ def test_explicit_workspace_and_graph_growth():
 
 
 def test_epoch_wraparound_resets_carry_words():
-    """the 32-bit launch epoch wraps after 2^32 launches of a workspace.  Put the epoch
-    just before the wrap and fill the carry words with words tagged 1..3 (what launches 2^32 ago
-    would have left): the wrap launch zeroes the words first, so no stale word validates."""
+    """the launch epoch in the carry tags wraps.  Tags are [20-bit epoch | 12-bit ring lap]
+    with the epoch part cycling 1..2^20-1; put the epoch two launches before a restart and fill the
+    carry ring with words carrying the tags the launches AFTER the restart will use (what launches
+    2^20-1 earlier would have left): the restart launch zeroes the ring first, so none validates."""
     S = sam()
     dc = S.SAM_I64
     n = 1 << 21
@@ -326,18 +327,21 @@ def test_epoch_wraparound_resets_carry_words():
     ws = torch.zeros(wsb // 8, dtype=torch.int64, device="cuda")
     carry = ws[1024 // 8:]
     stale = torch.randint(0, 1 << 31, (carry.numel(),), dtype=torch.int64, device="cuda")
-    carry.copy_(stale | (torch.randint(1, 4, (carry.numel(),), dtype=torch.int64, device="cuda") << 32))
+    ep_part = torch.randint(2, 5, (carry.numel(),), dtype=torch.int64, device="cuda")  # epochs 2..4, lap 0
+    carry.copy_(stale | ((ep_part << 12) << 32))
     hdr32 = ws[:4].view(torch.int32)
-    hdr32[3] = -3  # epoch word (offset 12) = 0xFFFFFFFD
+    period = (1 << 20) - 1
+    e0 = 5 * period - 2
+    hdr32[3] = e0  # epoch word (offset 12): tags 2^20-2, 2^20-1, then the restart (reset, 1), 2, 3, 4
     xn = synth.make(n, "i64", "uniform", seed=123)
     x = torch.from_numpy(xn).cuda()
-    for it in range(6):  # tags FE, FF, then the wrap launch (reset, tag 1), 2, 3, 4
+    for it in range(6):
         y = torch.empty_like(x)
         S.sam_scan_ws(dc, 2, 3, True, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(y.data_ptr()), n,
                       ctypes.c_void_p(ws.data_ptr()), wsb, S._stream_ptr())
         torch.cuda.synchronize()
         compare("i64", xn, y.cpu().numpy(), 2, 3, True)
-    assert int(hdr32[3].item()) == 4
+    assert int(hdr32[3].item()) == e0 + 6
 
 
 @pytest.mark.parametrize("name,k,s", [("f32", 1, 1), ("f64", 1, 1), ("f32", 2, 3), ("f64", 4, 4)])
