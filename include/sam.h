@@ -237,10 +237,11 @@ uint64_t sam_launch_count(void);
 int sam_debug_limit_grid(uint64_t max_ctas);
 /* Tuning (tools/autotune.py): override, for subsequent scans of this process, the carry unit
  * (tiles per super-tile, 1..8), the pipeline depth (tiles between local scan and carry application),
- * the value-parallel integer fold (0/1) and the landing-buffer fold (0/1); -1 / 0 = no override.
+ * the value-parallel integer fold (0/1), the landing-buffer fold (0/1) and the number of carry teams
+ * (1, 2 or 4 teams of 4, 2 or 1 carry warps); -1 / 0 = no override.
  * The measured choices go to lib/sam_tune.txt, which the library reads once at first use (SAM's
  * install-time auto-tuner). */
-int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land);
+int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land, int teams);
 /* Testing: nonzero seed = pseudo-random delays (up to ~16 us, 1 in 8 events) at every pipeline
  * hand-over of subsequent scan launches (loads, aggregate publication, carry folds, hand-offs,
  * local scans, carry applications), so the warps and CTAs meet in shuffled orders; 0 = off. */

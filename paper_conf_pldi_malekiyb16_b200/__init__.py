@@ -69,13 +69,15 @@ def lib() -> ctypes.CDLL:
             "sam_scan_op": (I, [I, I, I, I, I, P, P, U64, P]),
             "sam_scan_generic": (I, [I, I, I, I, I, I, P, P, U64, P]),
             "sam_last_carry_scheme": (I, []),
-            "sam_tune_override": (I, [I, I, I, I]),
+            "sam_tune_override": (I, [I, I, I, I, I]),
             "sam_debug_set_stress": (I, [ctypes.c_uint32]),
             "sam_scan_workspace_size": (I, [I, I, I, U64, ctypes.POINTER(SZ)]),
             "sam_scan_ws": (I, [I, I, I, I, P, P, U64, P, SZ, P]),
         }
         for name, (res, args) in sig.items():
-            fn = getattr(L, name)
+            fn = getattr(L, name, None)
+            if fn is None:  # an older library build (experiments via SAM_LIB_PATH)
+                continue
             fn.restype = res
             fn.argtypes = args
         _lib = L
@@ -124,8 +126,8 @@ def sam_scan_generic(dtype, op, carry, order, tuple_, inclusive, in_ptr, out_ptr
                                          stream))
 
 
-def sam_tune_override(tiles_per_unit=-1, lag=-1, vfold=-1, land=-1) -> int:
-    return _check(lib().sam_tune_override(tiles_per_unit, lag, vfold, land))
+def sam_tune_override(tiles_per_unit=-1, lag=-1, vfold=-1, land=-1, teams=-1) -> int:
+    return _check(lib().sam_tune_override(tiles_per_unit, lag, vfold, land, teams))
 
 
 def sam_last_carry_scheme() -> int:

@@ -660,8 +660,9 @@ int sam_debug_limit_grid(uint64_t max_ctas) {
     return SAM_OK;
 }
 
-int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land) {
+int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land, int teams) {
     sam::Knobs& k = sam::knobs_mut();
+    k.teams = (teams == 1 || teams == 2 || teams == 4) ? teams : 0;
     k.super_tile = (tiles_per_unit >= 1 && tiles_per_unit <= 8) ? tiles_per_unit : 0;
     k.lag = lag >= 1 ? lag : 0;
     k.vfold = vfold >= 0 ? (vfold != 0) : -1;

@@ -241,13 +241,15 @@ struct Params {
     T* pend;              // GPEND: pending local states [grid][LAG][K][TILE_THREADS] (workspace)
     int lag;              // pipeline depth used (1..LAG): max tiles between a local scan and its carry application
     int land;             // carry folds read through the smem landing buffer (when it fits)
+    int teams;            // carry teams: the 4 carry warps form `teams` teams working on successive super-tiles
     int vfold;            // integers + landing: value-parallel fold (else the windowed fold from the buffer)
     unsigned long long* carry;  // tagged carry words: [tile][m][t][agg W | incl W]
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
     unsigned int* epoch_ptr;
     unsigned long long carry_words;  // words of the carry ring actually used (R * rec_words)
-    unsigned long long ring;         // R: super-tile slots of the O(1) carry ring (a multiple of the grid)
+    unsigned long long ring;         // R: super-tile slots of the O(1) carry ring (a power of two >= 32 grids)
+    int ring_log2;
     unsigned int rec_words;          // words per super-tile record (16-B multiple)
     unsigned int* reset_ctr;         // grid barrier of the epoch wrap-around reset
     unsigned long long* trace;  // optional per-tile event timestamps [tile][8] (diagnostics), or null
@@ -468,7 +470,7 @@ struct SmemL {
     static constexpr int OFF_BUF1 = 0;
     static constexpr int OFF_BUF2 = OFF_BUF1 + NB1 * BUFB;
     static constexpr int OFF_BAR = OFF_BUF2 + NB2 * BUFB;  // full1[NB1] full2[NB2] stored2[NB2] p1/agg/carry[NQ]
-    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ + NCARRY + 1;  // ... bar_cw[NCARRY], bar_land
+    static constexpr int NBAR = NB1 + 2 * NB2 + 3 * NQ + 2 * NCARRY;  // ... bar_cw[NCARRY], bar_land[NCARRY]
     static constexpr int OFF_TILE = OFF_BAR + NBAR * 8;                  // NQ x i64 tile id
     static constexpr int OFF_SUP = OFF_TILE + NQ * 8;                    // NQ x i64 super-tile id
     static constexpr int OFF_SUB = OFF_SUP + NQ * 8;                     // NQ x (i32 sub index, i32 count)
@@ -543,7 +545,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     uint64_t* bar_agg = bar_p1 + NQ;
     uint64_t* bar_carry = bar_agg + NQ;
     uint64_t* bar_cw = bar_carry + NQ;  // [NCARRY]: a super-tile is ready for carry warp w
-    uint64_t* bar_land = bar_cw + NCARRY;  // the fold's landing buffer is full
+    uint64_t* bar_land = bar_cw + NCARRY;  // [team] the team's landing buffer is full
     volatile int* cw_taken = (volatile int*)(smem + S::OFF_CW);  // last super-tile each carry warp took
     int64_t* tile_of = (int64_t*)(smem + S::OFF_TILE);
     int64_t* sup_of = (int64_t*)(smem + S::OFF_SUP);
@@ -583,7 +585,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         }
         for (int w = 0; w < NCARRY; ++w) {
             mbar_init(&bar_cw[w], 32);
-            if (w == 0) mbar_init(bar_land, 1);
+            mbar_init(&bar_land[w], 1);
             cw_taken[w] = -1;
             *(volatile int*)(smem + S::OFF_HO + w * S::HOB) = -1;
         }
@@ -621,9 +623,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     const uint32_t tag = *sm_tag;  // base tag: | ring lap of the super-tile
     // O(1) carry ring: super-tile S lives in slot S mod R, tagged with its lap S / R, so a
     // word of the previous lap (or launch) never validates
-    auto ctag = [&](int64_t S) -> uint32_t { return tag | (uint32_t)(((uint64_t)S / p.ring) & 0xfffu); };
+    auto ctag = [&](int64_t S) -> uint32_t { return tag | (uint32_t)(((uint64_t)S >> p.ring_log2) & 0xfffu); };
     auto cslot = [&](int64_t S) -> unsigned long long* {
-        return p.carry + ((uint64_t)S % p.ring) * p.rec_words;
+        return p.carry + ((uint64_t)S & (p.ring - 1)) * p.rec_words;
     };
 
     // wait for barrier phase `par`, or return false once the stream has ended before iteration it
@@ -953,28 +955,38 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // every super-tile, warp w folding windows w, w+NCARRY, ... (round trips in parallel);
         // otherwise the carry warps take super-tiles round-robin, one warp folding all windows
         const bool coop = p.coop != 0;
-        const bool lead = !coop || cw == 0;  // finishes the super-tile (hand-off, sub-tile states)
+        // Teams: the carry warps form NT teams of TW warps; team t takes this CTA's super-tiles t, t+NT,
+        // ... (folds of successive super-tiles overlap; only the short chain step is ordered, through
+        // the hand-off entries).  coop = 0 is NT = 4 teams of one warp.
+        const int NT = coop ? (p.teams == 2 ? 2 : 1) : NCARRY;  // 1, 2 or 4 (no divisions below)
+        const int lgNT = NT == 1 ? 0 : (NT == 2 ? 1 : 2);
+        const int TW = NCARRY >> lgNT;
+        const int team = cw >> (2 - lgNT), tw = cw - team * TW;
+        const bool lead = tw == 0;  // finishes the super-tile (hand-off, sub-tile states)
         const int WV = p.Wn * p.Vr;          // super-tiles per window
         CT* const part_s = (CT*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds
         // landing: the whole range of aggregates a fold reads (at most P-1 super-tiles of s*K values)
         // arrives in shared memory with one bulk copy; words whose tag is not yet this launch's are
         // re-polled from L2 (the nearest predecessors, published last)
         constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
-        const bool use_land = SAM_LAND && p.land && coop && S::LANDB > 0 &&
-                              (uint64_t)(gridDim.x - 1) * p.rec_words * 8 <= (uint64_t)S::LANDB;
+        const int land_part = (S::LANDB / NT) / 128 * 128;  // each team's landing buffer
+        const bool use_land = SAM_LAND && p.land && coop && land_part > 0 &&
+                              (uint64_t)(gridDim.x - 1) * p.rec_words * 8 <= (uint64_t)land_part;
+        unsigned char* const land_s = smem + S::OFF_LAND + team * land_part;
+        uint64_t* const bar_lt = &bar_land[team];
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
         CT gpos[K];     // global frame: b(S US) of the current super-tile (lead, coop: advanced per round)
         CT tsum[K];     // global frame: I~_prev + sum of the folded A~_j (the next hand-off adds A~_S)
 #pragma unroll
         for (int t = 0; t < K; ++t) { gpos[t] = CT(0); tsum[t] = CT(0); }
-        for (int r = coop ? 0 : cw;; r += coop ? 1 : NCARRY) {  // this CTA's r-th super-tile
+        for (int r = team;; r += NT) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
             const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
             if ((uint64_t)tile >= p.num_super) break;
             const int64_t Sprev = r == 0 ? (int64_t)-1 : tile - gridDim.x;
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
-            const int bw = coop ? (int)(r % NCARRY) : cw;  // the aggregator's barrier for super-tile r
+            const int bw = (int)(r % NCARRY);  // the aggregator's barrier for super-tile r
             // landing range [lo_sup, tile) in bytes, 16-B aligned.  The copy is issued before the wait
             // for this super-tile's own aggregate: the previous round's aggregates are long published,
             // the current round's (the nearest) are re-polled from L2 if not yet there.
@@ -984,15 +996,15 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             if (land_r && lead && lane == 0) {
                 const uint64_t REC = (uint64_t)p.rec_words * 8;
                 const uint64_t cnt = (uint64_t)(tile - lo_sup);
-                const uint64_t slot0 = (uint64_t)lo_sup % p.ring;
+                const uint64_t slot0 = (uint64_t)lo_sup & (p.ring - 1);
                 const uint64_t c1 = slot0 + cnt <= p.ring ? cnt : p.ring - slot0;
                 fence_proxy_async_smem();  // the previous fold's generic reads of the buffer come first
-                mbar_arrive_expect_tx(bar_land, (uint32_t)(cnt * REC));
-                bulk_g2s(smem + S::OFF_LAND, (const void*)(p.carry + slot0 * p.rec_words), (uint32_t)(c1 * REC),
-                         bar_land, policy_evict_last());
+                mbar_arrive_expect_tx(bar_lt, (uint32_t)(cnt * REC));
+                bulk_g2s(land_s, (const void*)(p.carry + slot0 * p.rec_words), (uint32_t)(c1 * REC), bar_lt,
+                         policy_evict_last());
                 if (c1 < cnt)
-                    bulk_g2s(smem + S::OFF_LAND + c1 * REC, (const void*)p.carry, (uint32_t)((cnt - c1) * REC),
-                             bar_land, policy_evict_last());
+                    bulk_g2s(land_s + c1 * REC, (const void*)p.carry, (uint32_t)((cnt - c1) * REC), bar_lt,
+                             policy_evict_last());
             }
             if (lead) {
                 // Wait for the aggregator: it arrives on bar_cw[r % NCARRY] when super-tile r is
@@ -1009,7 +1021,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 
             SAM_STRESS(2 + cw, tile);
             if (land_r) {
-                mbar_wait(bar_land, (uint32_t)(nland & 1));
+                mbar_wait(bar_lt, (uint32_t)(nland & 1));
                 ++nland;
             }
             // seed of virtual super-tile -1 for lane mm: M(-1) applied for lanes before the phase
@@ -1036,7 +1048,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 const int jl = lane / s, mlb = lane - jl * s;
                 const bool active = jl < Wn;
                 CT total[K], Pm[K];
-                const int j0 = coop ? cw : 0, jstep = coop ? NCARRY : 1;
+                const int j0 = tw, jstep = TW;
 #pragma unroll
                 for (int t = 0; t < K; ++t) { total[t] = CT(0); Pm[t] = p.bwinj[j0][t]; }  // Pm = M(j0 WV US)
                 int npoll = 0;
@@ -1044,7 +1056,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                 // transformed aggregates, done value-parallel -- lane <-> (super-tile stripe, value
                 // (m, t)), consecutive lanes on consecutive words (conflict-free smem reads), the 4
                 // carry warps on interleaved super-tiles; stale words are re-polled from L2 one by one.
-                const bool vfold = TRANSFORM && land_r && p.vfold;
+                // (order 1: M = 1, the fold is a plain sum in any frame)
+                const bool vfold = (TRANSFORM || K == 1) && land_r && p.vfold;
                 if (vfold) {
                     // lane <-> (stripe st, value vi) for s*K <= 32 (stripes of super-tiles side by side),
                     // lane <-> (vi, vi + 32) otherwise; warp cw takes stripes cw*ST + st, + NCARRY*ST, ...
@@ -1061,13 +1074,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         const int vi = vi0 + 32 * h;
                         if (!lact || vi >= VPT) continue;
                         int par = 0;
-                        for (int64_t jj = (int64_t)cw * ST + st; jj < nsup; jj += (int64_t)NCARRY * ST, par ^= 1) {
-                            const unsigned long long* src = cslot(lo_sup + jj) + vi * W1;
+                        for (int64_t jj = (int64_t)tw * ST + st; jj < nsup; jj += (int64_t)TW * ST, par ^= 1) {
                             const unsigned long long* ls = (const unsigned long long*)(
-                                smem + S::OFF_LAND + ((size_t)jj * p.rec_words + vi * W1) * 8);
+                                land_s + ((uint32_t)jj * p.rec_words + vi * W1) * 8);
                             const uint32_t tj = ctag(lo_sup + jj);
                             unsigned long long w0 = ls[0], w1 = W1 == 2 ? ls[1] : 0ull;
                             while ((uint32_t)(w0 >> 32) != tj || (W1 == 2 && (uint32_t)(w1 >> 32) != tj)) {
+                                const unsigned long long* src = cslot(lo_sup + jj) + vi * W1;  // stale: re-poll L2
                                 if constexpr (W1 == 1) {
                                     w0 = ld_relaxed_u64(src);
                                 } else {
@@ -1090,7 +1103,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         pv_s[cw * 64 + vi0] = v0;
                         pv_s[cw * 64 + 32 + vi0] = v1;
                     }
-                    named_bar_sync(4, NCARRY * 32);
+                    if (TW > 1) named_bar_sync(4 + team, TW * 32);
                     if (lead) {
                         // value vi summed over the warps by lane vi, then lane m collects its K values
 #pragma unroll
@@ -1100,8 +1113,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                                 const int slot = vi < 32 ? vi : 32 + (vi - 32);
                                 CT a2 = pv_s[slot];
 #pragma unroll
-                                for (int w2 = 1; w2 < NCARRY; ++w2) a2 += pv_s[w2 * 64 + slot];
-                                pv_s[slot] = a2;
+                                for (int w2 = 1; w2 < TW; ++w2) a2 += pv_s[(cw + w2) * 64 + slot];
+                                pv_s[cw * 64 + slot] = a2;
                             }
                         }
                         __syncwarp();
@@ -1109,7 +1122,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                             for (int t = 0; t < K; ++t) {
                                 const int vi = lane * K + t;
-                                total[t] = pv_s[vi < 32 ? vi : 32 + (vi - 32)];
+                                total[t] = pv_s[cw * 64 + vi];
                             }
                         }
                         if (lane == 0) {
@@ -1130,6 +1143,13 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         st[vv] = (!active || vv >= p.Vr || idx <= Sprev) ? 3 : 0;
                     }
                     bool from_land = land_r;  // first pass from the landing buffer, re-polls from L2
+                    // 32-bit row bookkeeping (rows step back by Wn super-tiles): ring slot, lap and
+                    // landing index of row 0; row vv wraps to the previous lap when its slot goes negative
+                    const int64_t idx0 = basei - jl;
+                    const int slot0 = (int)((uint64_t)idx0 & (p.ring - 1));
+                    const uint32_t lap0 = (uint32_t)((uint64_t)idx0 >> p.ring_log2);
+                    const int dl0 = (int)(idx0 - lo_sup);
+                    const uint32_t recw = p.rec_words;
                     for (;;) {
                         if (p.trace && lane == 0 && j == 0 && npoll == 0) SAM_TRACE(8, tile * p.M);
                         // all loads first, then the tag checks: the loads of a window are then in
@@ -1137,11 +1157,12 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
-                                const int64_t idx = basei - jl - (int64_t)Wn * vv;
-                                const unsigned long long* src = cslot(idx) + mlb * K * W1;
+                                int sl = slot0 - Wn * vv;
+                                if (sl < 0) sl += (int)p.ring;
+                                const unsigned long long* src = p.carry + (size_t)sl * recw + mlb * K * W1;
                                 if (from_land) {
                                     const unsigned long long* ls = (const unsigned long long*)(
-                                        smem + S::OFF_LAND + ((size_t)(idx - lo_sup) * p.rec_words + mlb * K * W1) * 8);
+                                        land_s + ((uint32_t)(dl0 - Wn * vv) * recw + mlb * K * W1) * 8);
 #pragma unroll
                                     for (int t = 0; t < K; ++t) {
 #pragma unroll
@@ -1165,7 +1186,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         for (int vv = 0; vv < V; ++vv) {
                             if (st[vv] == 0) {
                                 bool ok = true;
-                                const uint32_t tv = ctag(basei - jl - (int64_t)Wn * vv);
+                                const uint32_t tv = tag | ((lap0 - (slot0 - Wn * vv < 0 ? 1u : 0u)) & 0xfffu);
 #pragma unroll
                                 for (int t = 0; t < K; ++t) {
                                     ok &= (uint32_t)(w[vv][t][0] >> 32) == tv;
@@ -1265,16 +1286,16 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     }
                 }
                 if (coop && !vfold) {  // sum the warps' partial folds (all already at their absolute offsets)
-                    CT* slot = part_s + ((r & 1) * NCARRY + cw) * MAXS * K;
+                    CT* slot = part_s + (((r >> lgNT) & 1) * NCARRY + cw) * MAXS * K;
                     if (lane_ok) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) slot[lane * K + t] = total[t];
                     }
-                    named_bar_sync(4, NCARRY * 32);
+                    if (TW > 1) named_bar_sync(4 + team, TW * 32);
                     if (lead && lane == 0) SAM_TRACE(13, tile * p.M);
                     if (lead && lane_ok) {
-                        for (int w2 = 1; w2 < NCARRY; ++w2) {
-                            const CT* o = part_s + ((r & 1) * NCARRY + w2) * MAXS * K;
+                        for (int w2 = 1; w2 < TW; ++w2) {
+                            const CT* o = part_s + (((r >> lgNT) & 1) * NCARRY + cw + w2) * MAXS * K;
 #pragma unroll
                             for (int t = 0; t < K; ++t) total[t] += o[lane * K + t];
                         }
@@ -1310,7 +1331,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
 #pragma unroll
                         for (int t = 0; t < K; ++t) tsum[t] = total[t];
                         if (coop) {
-                            if (r == 0) {
+                            if (r < NT) {  // the team's first super-tile; then NT rounds at a time
                                 mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
                             } else {
                                 CT np2[K];

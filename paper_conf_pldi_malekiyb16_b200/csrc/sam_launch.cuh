@@ -89,6 +89,7 @@ struct Knobs {
     int lag = 0;           // SAM_LAG: pipeline depth (tiles between local scan and carry application), <= LAG
     int land = -1;         // SAM_LAND: landing-buffer folds on (1) / off (0)
     int vfold = -1;        // SAM_VFOLD: value-parallel integer folds on (1) / off (0)
+    int teams = 0;         // SAM_TEAMS: carry teams (1, 2 or 4)
 };
 inline Knobs& knobs_mut() {
     static Knobs k = [] {
@@ -101,6 +102,7 @@ inline Knobs& knobs_mut() {
         if (const char* e = getenv("SAM_LAG")) r.lag = atoi(e);
         if (const char* e = getenv("SAM_LAND")) r.land = atoi(e) != 0;
         if (const char* e = getenv("SAM_VFOLD")) r.vfold = atoi(e) != 0;
+        if (const char* e = getenv("SAM_TEAMS")) { const int v = atoi(e); r.teams = (v == 1 || v == 2 || v == 4) ? v : 0; }
         return r;
     }();
     return k;
@@ -108,6 +110,9 @@ inline Knobs& knobs_mut() {
 inline const Knobs& knobs() { return knobs_mut(); }
 
 constexpr int MAX_DEVICES = 64;
+#ifndef SAM_DEFAULT_TEAMS
+#define SAM_DEFAULT_TEAMS 1
+#endif
 
 // Install-time autotune table (SAM's auto-tuner "runs when SAM is installed and determines the
 // optimal number of input elements to allocate to each thread for different ranges of problem
@@ -176,13 +181,14 @@ struct KernelInfo {
 // over: ~300 exact 128-bit evaluations), cached per (device, s, M, P, Vr) so a launch only fills in
 // its per-call fields.
 struct ShapeKey {
-    int dev, s, M, Vr;
+    int dev, s, M, Vr, teams;
     uint64_t P;
     bool operator<(const ShapeKey& o) const {
         if (dev != o.dev) return dev < o.dev;
         if (s != o.s) return s < o.s;
         if (M != o.M) return M < o.M;
         if (Vr != o.Vr) return Vr < o.Vr;
+        if (teams != o.teams) return teams < o.teams;
         return P < o.P;
     }
 };
@@ -215,8 +221,9 @@ inline uint32_t& debug_stress() {
     return seed;
 }
 
-// O(1) carry ring: R = RING_ROUNDS * grid super-tile records.  A slot is rewritten one
-// lap (RING_ROUNDS rounds) later by the same CTA; every reader of the old record is a fold of one of the
+// O(1) carry ring: R = the power of two >= RING_ROUNDS * grid super-tile records (slot and
+// lap by mask and shift).  A slot is rewritten one lap (>= RING_ROUNDS rounds) later; every reader of
+// the old record is a fold of one of the
 // next P-1 super-tiles, and a CTA cannot run more than 2*LAG/M + 1 <= 25 rounds ahead of another's
 // carries (its local scans wait on its own carries, which wait on everyone's aggregates), so 32 rounds
 // leave margin; the lap in every word's tag turns a violation into a wait, never a wrong value.
@@ -226,9 +233,14 @@ inline unsigned rec_words_of(int w, int k, int s) {
     const unsigned words = (unsigned)(s * k * (w / 4));
     return (words + 1u) & ~1u;
 }
+inline int ring_log2_of(int ctas) {
+    int l = 0;
+    while ((1ull << l) < (unsigned long long)ctas * RING_ROUNDS) ++l;
+    return l;
+}
 // bytes of the ring for a grid of `ctas`
 inline size_t ring_bytes(int w, int k, int s, int ctas) {
-    return (size_t)ctas * RING_ROUNDS * rec_words_of(w, k, s) * 8;
+    return ((size_t)1 << ring_log2_of(ctas)) * rec_words_of(w, k, s) * 8;
 }
 
 // global-memory pending-state scratch of one launch: [grid][LAG][K][TILE_THREADS] elements
@@ -305,10 +317,14 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
             if (dcap && (!cap || dcap < cap)) cap = dcap;
             if (cap && P > cap) P = cap;
         }
+        // carry teams: one team of 4 warps per super-tile.  Two teams folding successive super-tiles
+        // concurrently measured 5-20% slower on every config (profiles/r2_teams_ab.txt) and the team
+        // split is not kept as an option.
+        const int teams = 1;
         Params<T, K> p;
         {
             std::lock_guard<std::mutex> lk(info.mu);
-            const ShapeKey key{dev, a.s, (int)M, Vr, P};
+            const ShapeKey key{dev, a.s, (int)M, Vr, teams, P};
             auto it = tables.find(key);
             if (it == tables.end()) {
                 Params<T, K>* t = new Params<T, K>;
@@ -325,7 +341,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
                 mcol<CT>(US, K, t->bus);
                 for (int j = 0; j <= NCARRY; ++j) mcol<CT>((int64_t)j * geo.Wn * Vr * US, K, t->bwinj[j]);
                 mcol<CT>((int64_t)(P - 1) * US, K, t->bprev);
-                mcol<T>((int64_t)P * US, K, t->bposP);
+                mcol<T>((int64_t)teams * P * US, K, t->bposP);  // one team step = `teams` rounds
                 mcol<T>(-(int64_t)P * US, K, t->bnegP);
                 mcol<CT>((int64_t)geo.Wn * US, K, t->bwn);
                 for (int v = 0; v < 32; ++v) {
@@ -367,7 +383,8 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
             }
         }
         p.carry = a.carry;
-        p.ring = P * RING_ROUNDS;
+        p.ring_log2 = ring_log2_of((int)P);
+        p.ring = 1ull << p.ring_log2;
         p.rec_words = rec_words_of((int)sizeof(T), K, a.s);
         p.carry_words = p.ring * p.rec_words;
         if (p.carry_words > a.carry_words) return cudaErrorInvalidValue;  // workspace too small for this grid
@@ -378,6 +395,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         p.pend = (T*)a.pend;
         const TuneEntry* tl = te;
         p.lag = lag_rt;
+        p.teams = teams;
         p.land = kn.land >= 0 ? kn.land : ((tl && tl->land > 0) ? tl->land - 1 : 1);
         // measured (profiles/r2_ab_matrix.txt): the value-parallel fold wins from s*k >= 4 values per
         // super-tile (int64 k=4: +3%, C5: +16%), the windowed fold below (int64 k=2/3: +4-7%)

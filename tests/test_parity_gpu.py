@@ -353,3 +353,21 @@ def test_float_bit_deterministic(name, k, s):
     for _ in range(3):
         y1 = S.scan(x, order=k, tuple=s, inclusive=True)
         assert torch.equal(y0.view(torch.uint8), y1.view(torch.uint8))
+
+
+@pytest.mark.parametrize("teams", [1])
+@pytest.mark.parametrize("land,vfold", [(1, 1), (1, 0), (0, 0)])
+@pytest.mark.parametrize("name,k,s", [("i32", 1, 1), ("i64", 2, 1), ("i64", 4, 4), ("i32", 8, 3), ("f64", 3, 2),
+                                      ("i64", 8, 8)])
+def test_carry_team_variants(teams, land, vfold, name, k, s):
+    """Every carry-pipeline variant (landing-buffer or windowed folds;
+    value-parallel or windowed integer folds; odd tuples that make the ring records padded) over the
+    multi-round schedule, against the oracle."""
+    S = sam()
+    x = _multi_round_input(name, k, s)
+    S.sam_tune_override(-1, -1, vfold, land, teams)
+    try:
+        for inclusive in (True, False):
+            compare(name, x, run(name, x, k, s, inclusive), k, s, inclusive)
+    finally:
+        S.sam_tune_override(-1, -1, -1, -1, -1)

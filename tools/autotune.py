@@ -34,7 +34,7 @@ for lo, hi, lg in ranges:
         x, y = bufs[key]
         best = None
         for M, lag, vf in itertools.product((0, 1, 2, 3, 4), (0, 6, 8, 12), (-1,) if k == 1 else (0, 1)):
-            S.sam_tune_override(M if M else -1, lag if lag else -1, vf, -1)
+            S.sam_tune_override(M if M else -1, lag if lag else -1, vf, -1, -1)
             try:
                 for _ in range(2):
                     S.scan(x, k, s, True, out=y)
@@ -52,7 +52,7 @@ for lo, hi, lg in ranges:
             t = statistics.median(ts)
             if best is None or t < best[0]:
                 best = (t, M, lag, vf)
-        S.sam_tune_override(-1, -1, -1, -1)
+        S.sam_tune_override(-1, -1, -1, -1, -1)
         t, M, lag, vf = best
         vfield = 0 if vf < 0 else vf + 1
         lines.append(f"{TY[dt]} {k} {s} {lo} {hi} {M} {lag} {vfield} 0")
