@@ -242,6 +242,9 @@ int sam_debug_limit_grid(uint64_t max_ctas);
  * The measured choices go to lib/sam_tune.txt, which the library reads once at first use (SAM's
  * install-time auto-tuner). */
 int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land, int teams);
+/* Diagnostics: the launch shape of the last scan on this thread: out6 = {tiles per super-tile,
+ * pipeline depth, value-parallel fold, landing fold, grid CTAs, items per thread}. */
+int sam_debug_last_shape(int* out6);
 /* Testing: nonzero seed = pseudo-random delays (up to ~16 us, 1 in 8 events) at every pipeline
  * hand-over of subsequent scan launches (loads, aggregate publication, carry folds, hand-offs,
  * local scans, carry applications), so the warps and CTAs meet in shuffled orders; 0 = off. */

@@ -16,7 +16,7 @@ import os
 __all__ = [
     "SamError", "lib", "SAM_I32", "SAM_I64", "SAM_F32", "SAM_F64",
     "sam_scan", "sam_scan_seeded", "sam_scan_host", "sam_prepare", "sam_scan_workspace_size", "sam_scan_ws",
-    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_scan_op", "sam_scan_generic", "sam_last_carry_scheme", "sam_tune_override",
+    "sam_debug_limit_grid", "sam_debug_set_stress", "sam_scan_op", "sam_scan_generic", "sam_last_carry_scheme", "sam_tune_override", "sam_debug_last_shape",
     "scan_op", "SAM_U32", "SAM_U64", "SAM_OP", "SAM_CARRY", "sam_shard_payload_bytes",
     "sam_shard_state", "sam_shard_scan", "sam_fold_payloads_host", "sam_last_error", "sam_version",
     "sam_launch_count", "sam_release_workspaces", "sam_delta_encode", "sam_delta_encode_halo", "sam_delta_encode_host", "delta_encode_host", "scan", "delta_encode", "scan_host", "dtype_code", "LIB_PATH",
@@ -70,6 +70,7 @@ def lib() -> ctypes.CDLL:
             "sam_scan_generic": (I, [I, I, I, I, I, I, P, P, U64, P]),
             "sam_last_carry_scheme": (I, []),
             "sam_tune_override": (I, [I, I, I, I, I]),
+            "sam_debug_last_shape": (I, [ctypes.POINTER(ctypes.c_int)]),
             "sam_debug_set_stress": (I, [ctypes.c_uint32]),
             "sam_scan_workspace_size": (I, [I, I, I, U64, ctypes.POINTER(SZ)]),
             "sam_scan_ws": (I, [I, I, I, I, P, P, U64, P, SZ, P]),
@@ -128,6 +129,12 @@ def sam_scan_generic(dtype, op, carry, order, tuple_, inclusive, in_ptr, out_ptr
 
 def sam_tune_override(tiles_per_unit=-1, lag=-1, vfold=-1, land=-1, teams=-1) -> int:
     return _check(lib().sam_tune_override(tiles_per_unit, lag, vfold, land, teams))
+
+
+def sam_debug_last_shape() -> dict:
+    v = (ctypes.c_int * 6)()
+    _check(lib().sam_debug_last_shape(v))
+    return dict(zip(("M", "lag", "vfold", "land", "grid", "items"), list(v)))
 
 
 def sam_last_carry_scheme() -> int:

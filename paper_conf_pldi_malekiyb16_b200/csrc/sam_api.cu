@@ -670,6 +670,12 @@ int sam_tune_override(int tiles_per_unit, int lag, int vfold, int land, int team
     return SAM_OK;
 }
 
+int sam_debug_last_shape(int* out6) {
+    if (!out6) return fail(SAM_ERR_INVALID_ARG, "null output");
+    for (int i = 0; i < 6; ++i) out6[i] = sam::last_shape()[i];
+    return SAM_OK;
+}
+
 int sam_debug_set_stress(uint32_t seed) {
     sam::debug_stress() = seed;
     return SAM_OK;

@@ -216,6 +216,11 @@ inline uint64_t& debug_grid_cap(int dev) {
     static uint64_t cap[MAX_DEVICES] = {};
     return cap[dev];
 }
+// diagnostics: the shape of the last scan launch on this thread {M, lag, vfold, land, grid, ITEMS}
+inline int* last_shape() {
+    static thread_local int v[6] = {0, 0, 0, 0, 0, 0};
+    return v;
+}
 inline uint32_t& debug_stress() {
     static uint32_t seed = 0;
     return seed;
@@ -227,7 +232,10 @@ inline uint32_t& debug_stress() {
 // next P-1 super-tiles, and a CTA cannot run more than 2*LAG/M + 1 <= 25 rounds ahead of another's
 // carries (its local scans wait on its own carries, which wait on everyone's aggregates), so 32 rounds
 // leave margin; the lap in every word's tag turns a violation into a wait, never a wrong value.
-constexpr int RING_ROUNDS = 32;
+#ifndef SAM_RING_ROUNDS
+#define SAM_RING_ROUNDS 32
+#endif
+constexpr int RING_ROUNDS = SAM_RING_ROUNDS;
 // 64-bit words per super-tile record: s*k values of 1 or 2 words, padded to 16 B (bulk copies)
 inline unsigned rec_words_of(int w, int k, int s) {
     const unsigned words = (unsigned)(s * k * (w / 4));
@@ -397,9 +405,9 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         p.lag = lag_rt;
         p.teams = teams;
         p.land = kn.land >= 0 ? kn.land : ((tl && tl->land > 0) ? tl->land - 1 : 1);
-        // measured (profiles/r2_ab_matrix.txt): the value-parallel fold wins from s*k >= 4 values per
-        // super-tile (int64 k=4: +3%, C5: +16%), the windowed fold below (int64 k=2/3: +4-7%)
-        p.vfold = kn.vfold >= 0 ? kn.vfold : ((tl && tl->vfold > 0) ? tl->vfold - 1 : (a.s * K >= 4 ? 1 : 0));
+        // measured (profiles/r2_ab_ring.txt): with the ring the value-parallel fold wins or ties on every
+        // config (C2 +7%, int64 k=2 +10%, C5 +16%); the windowed fold stays for floats of order >= 2
+        p.vfold = kn.vfold >= 0 ? kn.vfold : ((tl && tl->vfold > 0) ? tl->vfold - 1 : 1);
         p.trace = a.trace;
         p.stress = debug_stress();
 
@@ -421,6 +429,10 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
             P = P - (P + 3) / 4;
             (simulated ? debug_grid_cap(dev) : grid_cap(dev)) = P;
             continue;
+        }
+        if (e == cudaSuccess) {
+            int* ls = last_shape();
+            ls[0] = p.M; ls[1] = p.lag; ls[2] = p.vfold; ls[3] = p.land; ls[4] = (int)P; ls[5] = ITEMS;
         }
         if (launches && e == cudaSuccess) ++*launches;
         return e != cudaSuccess ? e : cudaGetLastError();
