@@ -139,7 +139,8 @@ def cpu_model():
 # log2 n, order, tuple.  C3: int32/int64 orders 1..8; C4: int64 tuples 1..8 at orders 1, 2 and
 # fp32/fp64 tuples at order 1; C5: int64 order 4 tuple 4 at 2^30 (one GPU's weak-scaling share) and
 # at 2^33 (the strong-scaling total, > 2^32 elements, 128 GiB of HBM).
-SWEEP = ([(f"C3 i32 k={k}", "i32", 28, k, 1) for k in range(1, 9)] +
+SWEEP = ([("C1 i32 k=1 s=1 n=2^20 (L2-resident, launch-bound)", "i32", 20, 1, 1)] +
+         [(f"C3 i32 k={k}", "i32", 28, k, 1) for k in range(1, 9)] +
          [(f"C3 i64 k={k}", "i64", 28, k, 1) for k in range(1, 9)] +
          [(f"C4 i64 k={k} s={s}", "i64", 28, k, s) for k in (1, 2) for s in range(1, 9)] +
          [(f"C4 {d} k=1 s={s}", d, 28, 1, s) for d in ("f32", "f64") for s in range(1, 9)] +
@@ -187,6 +188,15 @@ def run_sweep(sam, synth, torch, peak, reps=5):
             torch.cuda.synchronize()
             memcpy_cache[key] = e0.elapsed_time(e1) / reps
         gbs = 2 * w * n / (ms * 1e-3) / 1e9
+        if logn <= 24:  # L2-resident: also the exclusive scan, and the per-launch time (launch-bound)
+            e0.record(st)
+            for _ in range(reps):
+                sam.sam_scan(dc, k, s, False, P(x), P(y), n, sp)
+            e1.record(st)
+            torch.cuda.synchronize()
+            out.append({"config": name + " exclusive", "n": n, "order": k, "tuple": s, "dtype": DTYPE_NAME[dt],
+                        "us_per_launch": e0.elapsed_time(e1) / reps * 1e3,
+                        "gvalues_s": n / (e0.elapsed_time(e1) / reps * 1e-3) / 1e9, "l2_resident": True})
         out.append({"config": name, "n": n, "order": k, "tuple": s, "dtype": DTYPE_NAME[dt],
                     "gvalues_s": n / (ms * 1e-3) / 1e9, "gbs": gbs, "ms": ms,
                     "frac_of_memcpy": memcpy_cache[key] / ms, "roofline_frac": gbs / peak,

@@ -487,7 +487,8 @@ struct SmemL {
     static constexpr int OFF_HO = OFF_BQ + 8 * K * (int)sizeof(T);       // [NCARRY] inclusive-state hand-off
     static constexpr int OFF_PART = (OFF_HO + NCARRY * HOB + 15) / 16 * 16;   // [2][NCARRY][MAXS][K]
     static constexpr int OFF_PV = OFF_PART + 2 * NCARRY * MAXS * K * (int)sizeof(CT);  // [NCARRY][64] value-parallel fold partials
-    static constexpr int OFF_EQ = OFF_PV + NCARRY * 64 * (int)sizeof(CT);                // [ELAG][TILE_THREADS][K]
+    static constexpr int OFF_GN = OFF_PV + NCARRY * 64 * (int)sizeof(CT);                // [2][K] next b(S US) (global frame)
+    static constexpr int OFF_EQ = OFF_GN + 2 * K * (int)sizeof(CT);                     // [ELAG][TILE_THREADS][K]
     static constexpr int BYTES0 = OFF_EQ + ELAG * TILE_THREADS * K * (int)sizeof(T);
     // carry-fold landing buffer: the P-1 aggregates a fold reads, pulled from L2 in ONE bulk copy
     // (whatever shared memory is left, up to 40 KB; the fold falls back to windowed loads if short)
@@ -1301,6 +1302,26 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
                     }
                 }
+                if (TRANSFORM && coop && TW > 1 && tw == 1) {
+                    // the next super-tile's b(S' US), S' = S + NT*P, for the lead (after the team barrier of
+                    // this super-tile, so the slot it fills is read only after the next one)
+                    if (r < NT) mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
+                    CT np2[K];
+#pragma unroll
+                    for (int d = 0; d < K; ++d) {
+                        CT acc2 = CT(0);
+#pragma unroll
+                        for (int e2 = 0; e2 <= d; ++e2) acc2 += gpos[e2] * p.bposP[d - e2];
+                        np2[d] = acc2;
+                    }
+#pragma unroll
+                    for (int d = 0; d < K; ++d) gpos[d] = np2[d];
+                    CT* gn = (CT*)(smem + S::OFF_GN) + (((r + NT) >> lgNT) & 1) * K;
+                    if (lane == 0) {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) gn[t] = np2[t];
+                    }
+                }
                 if (lead) {
                     // the CTA's own chain, kept to a few operations: C = F + M((S-1-Sprev) US) I_prev,
                     // I_prev = this CTA's inclusive state after Sprev (hand-off) or, for r = 0, the seed
@@ -1330,7 +1351,17 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
 #pragma unroll
                         for (int t = 0; t < K; ++t) tsum[t] = total[t];
-                        if (coop) {
+                        if (coop && TW > 1) {
+                            // b(S US): computed here for the team's first super-tile, afterwards ahead of
+                            // time by the team's second warp (off this serial path, see below)
+                            if (r < NT) {
+                                mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
+                            } else {
+                                const CT* gn = (const CT*)(smem + S::OFF_GN) + ((r >> lgNT) & 1) * K;
+#pragma unroll
+                                for (int t = 0; t < K; ++t) gpos[t] = gn[t];
+                            }
+                        } else if (coop) {
                             if (r < NT) {  // the team's first super-tile; then NT rounds at a time
                                 mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
                             } else {
