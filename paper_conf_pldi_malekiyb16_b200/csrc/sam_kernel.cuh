@@ -243,6 +243,8 @@ struct Params {
     int land;             // carry folds read through the smem landing buffer (when it fits)
     int teams;            // carry teams: the 4 carry warps form `teams` teams working on successive super-tiles
     int vfold;            // integers + landing: value-parallel fold (else the windowed fold from the buffer)
+    int dyn;              // dynamic claims: super-tiles taken from an atomic counter in claim order (else the
+                          // static schedule b, b+P, ...); the fold spans (own previous, S) whatever its length
     unsigned long long* carry;  // tagged carry words: [tile][m][t][agg W | incl W]
     unsigned long long* tile_ctr;
     unsigned int* done_ctr;
@@ -450,6 +452,17 @@ template <typename T> struct IsInt { static constexpr bool value = false; };
 template <> struct IsInt<uint32_t> { static constexpr bool value = true; };
 template <> struct IsInt<uint64_t> { static constexpr bool value = true; };
 
+// b_d(L) = C(L-1+d, d), d < K (first column of M(L)), lane d computing one binomial, broadcast to
+// the warp (all 32 lanes must call it)
+template <typename T, int K>
+__device__ __forceinline__ void mcol_warp(int64_t L, T (&b)[K]) {
+    const int lane = threadIdx.x & 31;
+    const int d = lane < K ? lane : 0;
+    const T mine = Arith<T>::binom(L - 1 + d, d);
+#pragma unroll
+    for (int t = 0; t < K; ++t) b[t] = __shfl_sync(0xffffffffu, mine, t);
+}
+
 // ------------------------------------------------------------------------------------------
 // shared-memory layout
 // ------------------------------------------------------------------------------------------
@@ -556,6 +569,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     volatile int* sm_end = (volatile int*)(smem + S::OFF_TAG + 4);
     volatile int* agg_done = (volatile int*)(smem + S::OFF_TAG + 8);  // iterations aggregated
     volatile int* lb_started = (volatile int*)(smem + S::OFF_TAG + 20);  // last super-tile whose fold began
+    volatile int* claimed = (volatile int*)(smem + S::OFF_TAG + 24);     // iterations claimed (dynamic claims)
     T* wq_all = (T*)(smem + S::OFF_WQ);
     T* la_all = (T*)(smem + S::OFF_LA);
     T* bt_s = (T*)(smem + S::OFF_BT);
@@ -601,6 +615,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         *agg_done = 0;
         *(volatile int*)(smem + S::OFF_TAG + 12) = 0;
         *lb_started = -1;
+        *claimed = 0;
     }
     for (int i = tid; i < K * 32; i += blockDim.x) bt_s[i] = (&p.bt[0][0])[i];
     for (int i = tid; i < K * 32; i += blockDim.x) bn_s[i] = (&p.bn[0][0])[i];
@@ -724,7 +739,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     (j1 < NB1 || mbar_test(&bar_p1[(j1 - NB1) % NQ], (uint32_t)(((j1 - NB1) / NQ) & 1))) &&
                     (j1 < PF || mbar_test(&bar_p1[(j1 - PF) % NQ], (uint32_t)(((j1 - PF) / NQ) & 1)))) {
                     if (cur_j == cur_cnt) {  // start the next super-tile
-                        cur_sup = (int64_t)blockIdx.x + (int64_t)nsup * gridDim.x;
+                        // static schedule: b, b+P, ...; dynamic: the next one in claim order
+                        cur_sup = p.dyn ? (int64_t)atomicAdd(p.tile_ctr, 1ull)
+                                        : (int64_t)blockIdx.x + (int64_t)nsup * gridDim.x;
                         ++nsup;
                         cur_j = 0;
                         cur_cnt = 0;
@@ -748,6 +765,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         SAM_STRESS(0, t);
                         load_tile(t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1], pol_keep);
                         ++j1;
+                        flag_st_rel(claimed, j1);  // tile_of / sup_of / sub_of of iteration j1-1 are set
                     }
                     continue;
                 }
@@ -772,6 +790,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const int64_t tile = tile_of[qs];
             const int64_t sup = sup_of[qs];
             const int jsub = sub_of[2 * qs], cnt = sub_of[2 * qs + 1];
+            if constexpr (TRANSFORM) {  // dynamic claims: b(-(S+1) US) of this super-tile, from its id
+                if (p.dyn && jsub == 0) mcol_warp<T, K>(-(sup + 1) * (int64_t)p.M * p.U, gneg);
+            }
             if (lane == 0) SAM_TRACE(2, tile);
             SAM_STRESS(1, tile);
             T* wq = wq_all + qs * S::WQ;
@@ -920,7 +941,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             __syncwarp();
             if (lane == 0) SAM_TRACE(3, tile);
             mbar_arrive(&bar_agg[qs]);
-            if (TRANSFORM && jsub == cnt - 1) {  // next super-tile of this CTA: one round further
+            if (TRANSFORM && !p.dyn && jsub == cnt - 1) {  // next super-tile of this CTA: one round further
                 T ng[K];
 #pragma unroll
                 for (int d = 0; d < K; ++d) {
@@ -971,8 +992,9 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // re-polled from L2 (the nearest predecessors, published last)
         constexpr uint64_t SUPB = (uint64_t)K * W1 * 8;  // bytes per (super-tile, lane)
         const int land_part = (S::LANDB / NT) / 128 * 128;  // each team's landing buffer
+        // (static schedule: every fold spans P-1 super-tiles; dynamic claims: checked per fold)
         const bool use_land = SAM_LAND && p.land && coop && land_part > 0 &&
-                              (uint64_t)(gridDim.x - 1) * p.rec_words * 8 <= (uint64_t)land_part;
+                              (p.dyn || (uint64_t)(gridDim.x - 1) * p.rec_words * 8 <= (uint64_t)land_part);
         unsigned char* const land_s = smem + S::OFF_LAND + team * land_part;
         uint64_t* const bar_lt = &bar_land[team];
         int nland = 0;  // landing copies consumed so far (mbarrier parity)
@@ -980,11 +1002,40 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         CT tsum[K];     // global frame: I~_prev + sum of the folded A~_j (the next hand-off adds A~_S)
 #pragma unroll
         for (int t = 0; t < K; ++t) { gpos[t] = CT(0); tsum[t] = CT(0); }
+        int64_t sprev_dyn = -1;  // dynamic claims: this CTA's previous super-tile
         for (int r = team;; r += NT) {  // this CTA's r-th super-tile
             const int i0 = r * p.M;       // its first iteration
-            const int64_t tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;  // global super-tile id
-            if ((uint64_t)tile >= p.num_super) break;
-            const int64_t Sprev = r == 0 ? (int64_t)-1 : tile - gridDim.x;
+            int64_t tile, Sprev;          // global super-tile id; this CTA's previous one (-1: none)
+            if (p.dyn) {
+                // the producer claims super-tiles in order: wait until it has taken this CTA's r-th
+                // (its id is then in sup_of), or the stream has ended before it
+                int st2 = 0;
+                if (lane == 0) {
+                    for (;;) {
+                        if (flag_ld_acq(claimed) > i0) { st2 = 1; break; }
+                        const int e = flag_ld(sm_end);
+                        if (e >= 0 && i0 >= e) break;
+                        __nanosleep(32);
+                    }
+                }
+                if (!__shfl_sync(0xffffffffu, st2, 0)) break;
+                tile = sup_of[i0 % NQ];
+                Sprev = sprev_dyn;
+                sprev_dyn = tile;
+                if constexpr (TRANSFORM) {
+                    // b(S US) for the lead's chain step, by the team's second warp while the fold runs
+                    if (coop && TW > 1 && tw == 1) {
+                        CT gp[K];
+                        mcol_warp<CT, K>(tile * (int64_t)p.M * p.U, gp);
+                        CT* gn = (CT*)(smem + S::OFF_GN) + (r & 1) * K;
+                        if (lane < K) gn[lane] = gp[lane];
+                    }
+                }
+            } else {
+                tile = (int64_t)blockIdx.x + (int64_t)r * gridDim.x;
+                if ((uint64_t)tile >= p.num_super) break;
+                Sprev = r == 0 ? (int64_t)-1 : tile - gridDim.x;
+            }
             const bool lane_ok = lane < s;
             const int ml = lane_ok ? lane : 0;
             const int bw = (int)(r % NCARRY);  // the aggregator's barrier for super-tile r
@@ -992,7 +1043,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             // for this super-tile's own aggregate: the previous round's aggregates are long published,
             // the current round's (the nearest) are re-polled from L2 if not yet there.
             const int64_t lo_sup = Sprev + 1;
-            const bool land_r = use_land && tile > lo_sup;
+            const bool land_r = use_land && tile > lo_sup &&
+                                (uint64_t)(tile - lo_sup) * p.rec_words * 8 <= (uint64_t)land_part;
             // landing offset of super-tile j: (j - lo_sup) * REC; the ring range may wrap: two copies
             if (land_r && lead && lane == 0) {
                 const uint64_t REC = (uint64_t)p.rec_words * 8;
@@ -1302,7 +1354,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
                     }
                 }
-                if (TRANSFORM && coop && TW > 1 && tw == 1) {
+                if (TRANSFORM && !p.dyn && coop && TW > 1 && tw == 1) {
                     // the next super-tile's b(S' US), S' = S + NT*P, for the lead (after the team barrier of
                     // this super-tile, so the slot it fills is read only after the next one)
                     if (r < NT) mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
@@ -1335,6 +1387,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         const CT* hv = (const CT*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB + 16);
 #pragma unroll
                         for (int t = 0; t < K; ++t) { pv[t] = hv[ml * K + t]; bcol[t] = p.bprev[t]; }
+                        if (!TRANSFORM && K > 1 && p.dyn)  // floats: span from the previous super-tile to S-1
+                            mcol<CT>((tile - 1 - Sprev) * (int64_t)p.M * p.U, K, bcol);
                         have = true;
                     } else if (p.seed) {
                         seed_of(ml, pv);
@@ -1351,7 +1405,15 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         }
 #pragma unroll
                         for (int t = 0; t < K; ++t) tsum[t] = total[t];
-                        if (coop && TW > 1) {
+                        if (p.dyn) {
+                            if (coop && TW > 1) {  // b(S US) from the team's second warp (above)
+                                const CT* gn = (const CT*)(smem + S::OFF_GN) + (r & 1) * K;
+#pragma unroll
+                                for (int t = 0; t < K; ++t) gpos[t] = gn[t];
+                            } else {
+                                mcol<CT>(tile * (int64_t)p.M * p.U, K, gpos);
+                            }
+                        } else if (coop && TW > 1) {
                             // b(S US): computed here for the team's first super-tile, afterwards ahead of
                             // time by the team's second warp (off this serial path, see below)
                             if (r < NT) {
@@ -1404,7 +1466,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             const T* la = la_all + (il % NQ) * S::LA;    // super-tile aggregate
             // hand the inclusive state M(M US) C + A to this CTA's next super-tile (in order
             // r-1 -> r: slot r % NCARRY is free once r-1's entry exists, r-1 having waited for r-2 ...)
-            if ((uint64_t)tile + gridDim.x < p.num_super) {
+            if (p.dyn || (uint64_t)tile + gridDim.x < p.num_super) {  // (dynamic: a next one may follow)
                 if (r > 0) {
                     const volatile int* rt = (const volatile int*)(smem + S::OFF_HO + ((r - 1) % NCARRY) * S::HOB);
                     while (flag_ld_acq(rt) != r - 1) __nanosleep(20);

@@ -90,6 +90,7 @@ struct Knobs {
     int land = -1;         // SAM_LAND: landing-buffer folds on (1) / off (0)
     int vfold = -1;        // SAM_VFOLD: value-parallel integer folds on (1) / off (0)
     int teams = 0;         // SAM_TEAMS: carry teams (1, 2 or 4)
+    int dyn = -1;          // SAM_DYN: dynamic (claim-order) super-tile schedule (1) or static b, b+P, ... (0)
 };
 inline Knobs& knobs_mut() {
     static Knobs k = [] {
@@ -102,6 +103,7 @@ inline Knobs& knobs_mut() {
         if (const char* e = getenv("SAM_LAG")) r.lag = atoi(e);
         if (const char* e = getenv("SAM_LAND")) r.land = atoi(e) != 0;
         if (const char* e = getenv("SAM_VFOLD")) r.vfold = atoi(e) != 0;
+        if (const char* e = getenv("SAM_DYN")) r.dyn = atoi(e) != 0;
         if (const char* e = getenv("SAM_TEAMS")) { const int v = atoi(e); r.teams = (v == 1 || v == 2 || v == 4) ? v : 0; }
         return r;
     }();
@@ -110,6 +112,9 @@ inline Knobs& knobs_mut() {
 inline const Knobs& knobs() { return knobs_mut(); }
 
 constexpr int MAX_DEVICES = 64;
+#ifndef SAM_DEFAULT_DYN
+#define SAM_DEFAULT_DYN 0
+#endif
 #ifndef SAM_DEFAULT_TEAMS
 #define SAM_DEFAULT_TEAMS 1
 #endif
@@ -408,6 +413,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         // measured (profiles/r2_ab_ring.txt): with the ring the value-parallel fold wins or ties on every
         // config (C2 +7%, int64 k=2 +10%, C5 +16%); the windowed fold stays for floats of order >= 2
         p.vfold = kn.vfold >= 0 ? kn.vfold : ((tl && tl->vfold > 0) ? tl->vfold - 1 : 1);
+        p.dyn = kn.dyn >= 0 ? kn.dyn : SAM_DEFAULT_DYN;
         p.trace = a.trace;
         p.stress = debug_stress();
 

@@ -62,3 +62,22 @@ if len(first) > 2:
     e = tf[f]
     print(f"  lbstart->poll0 {q(us(e[:, 8] - e[:, 4]))}  poll0->lbdone {q(us(e[:, 10] - e[:, 8]))}  lbdone->barrier {q(us(e[:, 13] - e[:, 10]))}"
           f"  barrier->handoff {q(us(e[:, 14] - e[:, 13]))}  handoff->incl0 {q(us(e[:, 5] - e[:, 14]))}")
+# skew: when did the last aggregate a super-tile's fold needs (super-tiles S-P+1..S-1) appear, relative to
+# the super-tile's own last aggregate and to its fold start / end
+if len(first) > 2:
+    P = int(os.environ.get("P", "148"))
+    lastagg = t[last, 3]
+    ns = len(f)
+    need = np.full(ns, np.nan)
+    for i in range(ns):
+        lo = max(0, i - P + 1)
+        if i > lo: need[i] = np.nanmax(lastagg[lo:i])
+    e = tf[f]
+    print(f"skew: need-ownagg {q(us(need - lastagg))}  need-poll0 {q(us(need - e[:, 8]))}  lbdone-need {q(us(e[:, 10] - need))}")
+    # per-CTA progress spread: for each round, max - min of the super-tiles' own last aggregate
+    R = ns // P
+    if R > 2:
+        la = lastagg[:R * P].reshape(R, P)
+        print(f"round spread of own-agg (max-min over CTAs) {q(us(np.nanmax(la, 1) - np.nanmin(la, 1)))}")
+        d = np.diff(np.nanmedian(la, 1))
+        print(f"round period (median own-agg) {q(us(d))}")
