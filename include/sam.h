@@ -170,6 +170,36 @@ int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const v
 int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* all_payloads_host,
                            int rank, int nranks, void* seed_host);
 
+/* ---------------------------------------------------------------------------------------
+ * Block-cyclic multi-GPU scan: SAM's carry scheme with the GPUs as the
+ * persistent blocks ("each block ... only needs to read the local sums of the
+ * previous P-1 chunks and its own carry from the previous iteration").  The global array is cut
+ * into chunks of C elements; chunk c lives on rank c mod p, so round r holds chunks r*p .. r*p+p-1
+ * (one per rank).  Per round each rank (1) runs sam_shard_state on its chunk (global offset
+ * c*C) while the chunk stays in L2, (2) all ranks exchange the p payloads of the round, (3)
+ * sam_cyclic_fold gives the carry into its chunk, (4) sam_scan_seeded scans the chunk (its re-read
+ * an L2 hit), so each element costs one HBM read and one write on every GPU -- contiguous shards
+ * cost 1.5x that (state pass over the whole shard, then the scan).
+ *
+ * sam_cyclic_fold: `round_payloads` (device, nranks * sam_shard_payload_bytes, rank order) = the
+ * payloads of one round; `base_in` (device, [tuple][order], or NULL = zero state) = the state of
+ * every global lane before the round (the stream seed before round 0).  Writes `seed_out`
+ * (device, [tuple][order]) = base (+) payloads of ranks < rank, the carry operator (+) of
+ * DESIGN.md §2 applied in rank order (lanes absent from a chunk pass through), and, if `base_out`
+ * is not NULL, base (+) all nranks payloads = the next round's base.  base_out may alias base_in.
+ * Every rank folds the same bytes in the same order: the bases are bit-identical on all ranks
+ * (floats included).  Errors: UNSUPPORTED for order/tuple outside 1..8, INVALID_ARG for null
+ * payloads/seed_out or rank outside [0, nranks).  One one-warp kernel, asynchronous on `stream`.
+ * --------------------------------------------------------------------------------------- */
+int sam_cyclic_fold(sam_dtype dtype, int order, int tuple, const void* round_payloads, int rank,
+                    int nranks, const void* base_in, void* seed_out, void* base_out,
+                    sam_stream_t stream);
+
+/* The same fold on host buffers (CPU orchestration and tests). */
+int sam_cyclic_fold_host(sam_dtype dtype, int order, int tuple, const void* round_payloads_host,
+                         int rank, int nranks, const void* base_in_host, void* seed_out_host,
+                         void* base_out_host);
+
 /*
  * sam_delta_encode -- the k-th order, tuple-s difference sequence (delta ENCODER), the inverse of
  * the inclusive sam_scan with the same (order, tuple):

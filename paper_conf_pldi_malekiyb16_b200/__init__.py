@@ -57,6 +57,8 @@ def lib() -> ctypes.CDLL:
             "sam_shard_state": (I, [I, I, I, P, U64, U64, P, P]),
             "sam_shard_scan": (I, [I, I, I, I, P, P, U64, U64, P, I, I, P]),
             "sam_fold_payloads_host": (I, [I, I, I, P, I, I, P]),
+            "sam_cyclic_fold": (I, [I, I, I, P, I, I, P, P, P, P]),
+            "sam_cyclic_fold_host": (I, [I, I, I, P, I, I, P, P, P]),
             "sam_delta_encode": (I, [I, I, I, P, P, U64, P]),
             "sam_delta_encode_halo": (I, [I, I, I, P, P, U64, P, P]),
             "sam_delta_encode_host": (I, [I, I, I, P, P, U64, P]),
@@ -169,6 +171,18 @@ def sam_shard_scan(dtype, order, tuple_, inclusive, in_ptr, out_ptr, n_local, gl
 
 def sam_fold_payloads_host(dtype, order, tuple_, payloads_host_ptr, rank, nranks, seed_host_ptr) -> int:
     return _check(lib().sam_fold_payloads_host(dtype, order, tuple_, payloads_host_ptr, rank, nranks, seed_host_ptr))
+
+
+def sam_cyclic_fold(dtype, order, tuple_, round_payloads_ptr, rank, nranks, base_in_ptr, seed_out_ptr,
+                    base_out_ptr, stream=None) -> int:
+    return _check(lib().sam_cyclic_fold(dtype, order, tuple_, round_payloads_ptr, rank, nranks, base_in_ptr,
+                                        seed_out_ptr, base_out_ptr, stream))
+
+
+def sam_cyclic_fold_host(dtype, order, tuple_, round_payloads_host_ptr, rank, nranks, base_in_host_ptr,
+                         seed_out_host_ptr, base_out_host_ptr) -> int:
+    return _check(lib().sam_cyclic_fold_host(dtype, order, tuple_, round_payloads_host_ptr, rank, nranks,
+                                             base_in_host_ptr, seed_out_host_ptr, base_out_host_ptr))
 
 
 def sam_delta_encode(dtype, order, tuple_, in_ptr, out_ptr, n, stream=None) -> int:

@@ -103,15 +103,16 @@ SAM_HD uint64_t lane_len(uint64_t n, uint64_t g, int s, int m) {
     return i0 < n ? (n - 1 - i0) / (uint64_t)s + 1 : 0;
 }
 
-// Fold gathered shard payloads of ranks < rank into the seed of `rank`.
-// payload j: [u64 n_j][u64 g_j][values T [s][k]]  (stride = payload_bytes)
-// seed[m][t] = state of global lane m at its last element before shard `rank`.
+// Fold `count` consecutive payloads onto the state base_m of global lane m (null = zero state):
+// payload j: [u64 n_j][u64 g_j][values T [s][k]]  (stride = payload_bytes), each the zero-seeded
+// state of every lane at its last element in a stream of n_j elements at global offset g_j.
+// out_m[t] = state of lane m after the last of them.  out_m may alias base_m.
 template <typename T>
-SAM_HD void fold_payloads(const unsigned char* payloads, size_t payload_bytes, int rank, int k,
-                          int s, int m, T* seed_m) {
+SAM_HD void fold_payloads_from(const T* base_m, const unsigned char* payloads, size_t payload_bytes,
+                               int count, int k, int s, int m, T* out_m) {
     T S[MAXK], tmp[MAXK], b[MAXK];
-    for (int t = 0; t < k; ++t) S[t] = T(0);
-    for (int j = 0; j < rank; ++j) {
+    for (int t = 0; t < k; ++t) S[t] = base_m ? base_m[t] : T(0);
+    for (int j = 0; j < count; ++j) {
         const unsigned char* p = payloads + (size_t)j * payload_bytes;
         uint64_t nj = ((const uint64_t*)p)[0];
         uint64_t gj = ((const uint64_t*)p)[1];
@@ -122,7 +123,15 @@ SAM_HD void fold_payloads(const unsigned char* payloads, size_t payload_bytes, i
         mapply<T>(b, S, k, tmp);
         for (int t = 0; t < k; ++t) S[t] = tmp[t] + v[t];
     }
-    for (int t = 0; t < k; ++t) seed_m[t] = S[t];
+    for (int t = 0; t < k; ++t) out_m[t] = S[t];
+}
+
+// Fold gathered shard payloads of ranks < rank into the seed of `rank`.
+// seed[m][t] = state of global lane m at its last element before shard `rank`.
+template <typename T>
+SAM_HD void fold_payloads(const unsigned char* payloads, size_t payload_bytes, int rank, int k,
+                          int s, int m, T* seed_m) {
+    fold_payloads_from<T>(nullptr, payloads, payload_bytes, rank, k, s, m, seed_m);
 }
 
 }  // namespace sam

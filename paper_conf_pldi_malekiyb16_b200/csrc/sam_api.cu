@@ -278,6 +278,17 @@ int payload_init(sam_dtype dtype, void* payload, uint64_t n, uint64_t g, int k, 
     return e == cudaSuccess ? SAM_OK : cuda_fail(e, "payload init launch");
 }
 
+template <typename T>
+void cyclic_fold_host_t(const unsigned char* P, size_t pb, int rank, int nranks, int k, int s, const T* base_in,
+                        T* seed_out, T* base_out) {
+    for (int m = 0; m < s; ++m) {
+        T sd[sam::MAXK];
+        sam::fold_payloads_from<T>(base_in ? base_in + m * k : nullptr, P, pb, rank, k, s, m, sd);
+        if (base_out) sam::fold_payloads_from<T>(sd, P + (size_t)rank * pb, pb, nranks - rank, k, s, m, base_out + m * k);
+        for (int t = 0; t < k; ++t) seed_out[m * k + t] = sd[t];
+    }
+}
+// block-cyclic fold on host buffers (sam_cyclic_fold_host)
 int store_mode_for(const void* in, const void* out) {
     return ((((uintptr_t)in) ^ ((uintptr_t)out)) & 15) == 0 ? sam::STORE_BULK : sam::STORE_STRIPED;
 }
@@ -418,6 +429,43 @@ int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* al
             case SAM_F32: sam::fold_payloads<float>(P, pb, rank, order, tuple, m, (float*)seed_host + m * order); break;
             default: sam::fold_payloads<double>(P, pb, rank, order, tuple, m, (double*)seed_host + m * order); break;
         }
+    }
+    return SAM_OK;
+}
+
+int sam_cyclic_fold(sam_dtype dtype, int order, int tuple, const void* round_payloads, int rank, int nranks,
+                    const void* base_in, void* seed_out, void* base_out, sam_stream_t stream) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAM_ERR_INVALID_ARG, "rank/nranks out of range");
+    if (!round_payloads || !seed_out) return fail(SAM_ERR_INVALID_ARG, "null payloads or seed_out");
+    const size_t pb = sam_shard_payload_bytes(dtype, order, tuple);
+    cudaStream_t st = (cudaStream_t)stream;
+    uint64_t l = 0;
+    cudaError_t e;
+    switch (dtype) {
+        case SAM_I32: e = sam::launch_cyclic_fold<uint32_t>(round_payloads, pb, rank, nranks, order, tuple, base_in, seed_out, base_out, st, &l); break;
+        case SAM_I64: e = sam::launch_cyclic_fold<uint64_t>(round_payloads, pb, rank, nranks, order, tuple, base_in, seed_out, base_out, st, &l); break;
+        case SAM_F32: e = sam::launch_cyclic_fold<float>(round_payloads, pb, rank, nranks, order, tuple, base_in, seed_out, base_out, st, &l); break;
+        default: e = sam::launch_cyclic_fold<double>(round_payloads, pb, rank, nranks, order, tuple, base_in, seed_out, base_out, st, &l); break;
+    }
+    g_launches += l;
+    return e == cudaSuccess ? SAM_OK : cuda_fail(e, "cyclic fold launch");
+}
+
+int sam_cyclic_fold_host(sam_dtype dtype, int order, int tuple, const void* round_payloads_host, int rank,
+                         int nranks, const void* base_in_host, void* seed_out_host, void* base_out_host) {
+    int rc = validate_common(dtype, order, tuple);
+    if (rc) return rc;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAM_ERR_INVALID_ARG, "rank/nranks out of range");
+    if (!round_payloads_host || !seed_out_host) return fail(SAM_ERR_INVALID_ARG, "null buffer");
+    const size_t pb = sam_shard_payload_bytes(dtype, order, tuple);
+    const unsigned char* P = (const unsigned char*)round_payloads_host;
+    switch (dtype) {
+        case SAM_I32: cyclic_fold_host_t<uint32_t>(P, pb, rank, nranks, order, tuple, (const uint32_t*)base_in_host, (uint32_t*)seed_out_host, (uint32_t*)base_out_host); break;
+        case SAM_I64: cyclic_fold_host_t<uint64_t>(P, pb, rank, nranks, order, tuple, (const uint64_t*)base_in_host, (uint64_t*)seed_out_host, (uint64_t*)base_out_host); break;
+        case SAM_F32: cyclic_fold_host_t<float>(P, pb, rank, nranks, order, tuple, (const float*)base_in_host, (float*)seed_out_host, (float*)base_out_host); break;
+        default: cyclic_fold_host_t<double>(P, pb, rank, nranks, order, tuple, (const double*)base_in_host, (double*)seed_out_host, (double*)base_out_host); break;
     }
     return SAM_OK;
 }

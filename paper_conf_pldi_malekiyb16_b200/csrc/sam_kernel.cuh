@@ -2025,6 +2025,27 @@ __global__ void sam_fold_kernel(const unsigned char* payloads, size_t payload_by
     if (mm < s) fold_payloads<T>(payloads, payload_bytes, rank, k, s, mm, seed + (size_t)mm * k);
 }
 
+// Block-cyclic multi-GPU: SAM's carry scheme with the GPUs as the persistent
+// blocks.  `payloads` = the nranks chunk payloads of one round (rank order), base_in =
+// the state before the round (null: zero).  seed_out = base (+) payloads of ranks < rank (the carry
+// into this rank's chunk); base_out (optional) = base (+) all of them (the next round's base).
+// One thread per tuple lane; every rank folds the same bytes in the same order, so all ranks hold
+// bit-identical bases.
+template <typename T>
+__global__ void sam_cyclic_fold_kernel(const unsigned char* payloads, size_t payload_bytes, int rank, int nranks,
+                                       int k, int s, const T* base_in, T* seed_out, T* base_out) {
+    const int mm = threadIdx.x;
+    if (mm >= s) return;
+    T st[MAXK];
+    for (int t = 0; t < k; ++t) st[t] = base_in ? base_in[(size_t)mm * k + t] : T(0);
+    fold_payloads_from<T>(st, payloads, payload_bytes, rank, k, s, mm, st);
+    for (int t = 0; t < k; ++t) seed_out[(size_t)mm * k + t] = st[t];
+    if (base_out) {
+        fold_payloads_from<T>(st, payloads + (size_t)rank * payload_bytes, payload_bytes, nranks - rank, k, s, mm, st);
+        for (int t = 0; t < k; ++t) base_out[(size_t)mm * k + t] = st[t];
+    }
+}
+
 // Payload header + lanes with no element in the stream: final state = seed (or 0).
 template <typename T>
 __global__ void sam_payload_init_kernel(unsigned char* payload, uint64_t n, uint64_t g, int k, int s,

@@ -461,6 +461,16 @@ cudaError_t launch_fold(const void* payloads, size_t payload_bytes, int rank, in
 }
 
 template <typename T>
+cudaError_t launch_cyclic_fold(const void* payloads, size_t payload_bytes, int rank, int nranks, int k, int s,
+                               const void* base_in, void* seed_out, void* base_out, cudaStream_t st,
+                               uint64_t* launches) {
+    sam_cyclic_fold_kernel<T><<<1, 32, 0, st>>>((const unsigned char*)payloads, payload_bytes, rank, nranks, k, s,
+                                                (const T*)base_in, (T*)seed_out, (T*)base_out);
+    if (launches) ++*launches;
+    return cudaGetLastError();
+}
+
+template <typename T>
 cudaError_t launch_payload_init(void* payload, uint64_t n, uint64_t g, int k, int s, const void* seed,
                                 int write_header, void* final_state, cudaStream_t st, uint64_t* launches) {
     sam_payload_init_kernel<T><<<1, 64, 0, st>>>((unsigned char*)payload, n, g, k, s, (const T*)seed,
@@ -483,6 +493,8 @@ cudaError_t launch_payload_init(void* payload, uint64_t n, uint64_t g, int k, in
     template cudaError_t launch_scan_tk<T, 8>(const LaunchArgs&, uint64_t*);                           \
     template cudaError_t launch_fold<T>(const void*, size_t, int, int, int, void*, cudaStream_t,       \
                                         uint64_t*);                                                    \
+    template cudaError_t launch_cyclic_fold<T>(const void*, size_t, int, int, int, int, const void*, void*,   \
+                                               void*, cudaStream_t, uint64_t*);                        \
     template cudaError_t launch_payload_init<T>(void*, uint64_t, uint64_t, int, int, const void*, int, \
                                                 void*, cudaStream_t, uint64_t*);                       \
     }

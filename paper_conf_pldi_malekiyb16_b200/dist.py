@@ -26,8 +26,8 @@ import ctypes
 import torch
 import torch.distributed as dist
 
-from . import (SamError, _stream_ptr, delta_encode, dtype_code, sam_shard_payload_bytes, sam_shard_scan,
-               sam_shard_state)
+from . import (SamError, _stream_ptr, delta_encode, dtype_code, sam_cyclic_fold, sam_scan_seeded,
+               sam_shard_payload_bytes, sam_shard_scan, sam_shard_state)
 
 TAIL = 64  # elements each rank contributes to the halo exchange (>= max order*tuple = 64)
 
@@ -118,6 +118,189 @@ def scan_virtual_shards(x: torch.Tensor, bounds: list[int], order: int = 1, tupl
                        ctypes.c_void_p(out.data_ptr() + lo * w), hi - lo, lo,
                        ctypes.c_void_p(gathered.data_ptr()), r, p, st)
     return out
+
+
+# ----------------------------------------------------------------------------- block-cyclic (NEXT-1)
+# SAM's persistent-block carry scheme with the GPUs as the blocks.
+# Chunk c (C elements, global offset c*C) lives on rank c mod p; round r = chunks r*p .. r*p+p-1.
+# Per round a rank runs the state pass over its chunk (the chunk stays in L2), the p payloads of the
+# round are exchanged, sam_cyclic_fold turns the round's base state + the payloads of ranks < rank
+# into this chunk's seed (and the next round's base), and the seeded scan re-reads the chunk from
+# L2: one HBM read and one write per element on every GPU (contiguous shards: 1.5x that).
+def cyclic_chunks(n_total: int, chunk: int, nranks: int, rank: int) -> list[tuple[int, int, int]]:
+    """This rank's chunks in round order: (global offset, length, offset in the local buffer)."""
+    if chunk < 1 or nranks < 1 or not 0 <= rank < nranks:
+        raise SamError(-1, "chunk >= 1 and 0 <= rank < nranks required")
+    out, lo, r = [], 0, 0
+    while (r * nranks + rank) * chunk < n_total:
+        g0 = (r * nranks + rank) * chunk
+        ln = min(chunk, n_total - g0)
+        out.append((g0, ln, lo))
+        lo += ln
+        r += 1
+    return out
+
+
+def cyclic_rounds(n_total: int, chunk: int, nranks: int) -> int:
+    """Rounds of the block-cyclic schedule (every rank takes part in every round; a rank without a
+    chunk in the last round contributes an empty payload)."""
+    return -(-(-(-n_total // chunk)) // nranks) if n_total > 0 else 0
+
+
+def cyclic_local_len(n_total: int, chunk: int, nranks: int, rank: int) -> int:
+    return sum(ln for _, ln, _ in cyclic_chunks(n_total, chunk, nranks, rank))
+
+
+def to_cyclic(x: torch.Tensor, chunk: int, nranks: int, rank: int) -> torch.Tensor:
+    """This rank's block-cyclic local buffer (its chunks concatenated) from a global array."""
+    parts = [x[g0:g0 + ln] for g0, ln, _ in cyclic_chunks(x.numel(), chunk, nranks, rank)]
+    return torch.cat(parts) if parts else x[:0].clone()
+
+
+def from_cyclic(locals_: list, chunk: int, n_total: int) -> torch.Tensor:
+    """Reassemble the global array from every rank's block-cyclic local buffer."""
+    p = len(locals_)
+    out = torch.empty(n_total, dtype=locals_[0].dtype, device=locals_[0].device)
+    for g in range(p):
+        for g0, ln, lo in cyclic_chunks(n_total, chunk, p, g):
+            out[g0:g0 + ln] = locals_[g][lo:lo + ln]
+    return out
+
+
+def _cyclic_steps(x_local, out, order, tuple_, inclusive, chunk, n_total, rank, nranks, lookahead, st_obj,
+                  seed=None):
+    """The per-rank schedule as a generator.  It yields ("send", r, payload) once the state pass of
+    round r is issued and ("recv", r) when the fold of round r needs the gathered payloads (the
+    driver sends back a device tensor of nranks * payload_bytes, rank order).  The state passes run
+    up to `lookahead` rounds ahead of the folds, so the exchange of round r overlaps the state pass
+    of round r + 1 (at the price of lookahead + 1 chunks held in L2).  Every kernel goes on st_obj."""
+    dc = dtype_code(x_local.dtype)
+    pb = sam_shard_payload_bytes(dc, order, tuple_)
+    dev = x_local.device
+    w = x_local.element_size()
+    chunks = cyclic_chunks(n_total, chunk, nranks, rank)
+    R = cyclic_rounds(n_total, chunk, nranks)
+    st = _stream_ptr(st_obj)
+    nbuf = lookahead + 2
+    payloads = torch.empty(nbuf, pb, dtype=torch.uint8, device=dev)
+    k_s = order * tuple_
+    base = torch.zeros(k_s, dtype=x_local.dtype, device=dev)
+    if seed is not None:
+        base.copy_(seed.reshape(-1))
+    seedbuf = torch.empty(k_s, dtype=x_local.dtype, device=dev)
+    xp, op_ = x_local.data_ptr(), out.data_ptr()
+
+    def state(r):
+        pl = payloads[r % nbuf]
+        if r < len(chunks):
+            g0, ln, lo = chunks[r]
+        else:  # no chunk of this rank in round r: an empty payload (every lane passes through)
+            g0, ln, lo = (r * nranks + rank) * chunk, 0, 0
+        sam_shard_state(dc, order, tuple_, ctypes.c_void_p(xp + lo * w if ln else 0), ln, g0,
+                        ctypes.c_void_p(pl.data_ptr()), st)
+        return pl
+
+    for r in range(min(lookahead + 1, R)):
+        yield ("send", r, state(r))
+    for r in range(R):
+        gathered = yield ("recv", r)
+        sam_cyclic_fold(dc, order, tuple_, ctypes.c_void_p(gathered.data_ptr()), rank, nranks,
+                        ctypes.c_void_p(base.data_ptr()), ctypes.c_void_p(seedbuf.data_ptr()),
+                        ctypes.c_void_p(base.data_ptr()), st)
+        if r < len(chunks):
+            g0, ln, lo = chunks[r]
+            sam_scan_seeded(dc, order, tuple_, inclusive, ctypes.c_void_p(xp + lo * w),
+                            ctypes.c_void_p(op_ + lo * w), ln, g0, ctypes.c_void_p(seedbuf.data_ptr()), None, st)
+        if r + lookahead + 1 < R:
+            yield ("send", r + lookahead + 1, state(r + lookahead + 1))
+
+
+def scan_cyclic(x_local: torch.Tensor, order: int = 1, tuple: int = 1, inclusive: bool = True,
+                chunk: int = 1 << 22, n_total: int | None = None, group=None, out: torch.Tensor | None = None,
+                lookahead: int | None = None, stream=None) -> torch.Tensor:
+    """Scan of a global array held block-cyclically: this rank's `x_local` is the concatenation of
+    chunks rank, rank + p, rank + 2p, ... of `chunk` elements (to_cyclic).  One all-gather of p
+    payloads (<= 528 B each) per round -- the exchange step -- issued asynchronously so it overlaps
+    the next round's state pass; every arithmetic step runs in libsam.so kernels on `stream`."""
+    if not x_local.is_cuda or x_local.dim() != 1 or not x_local.is_contiguous():
+        raise SamError(-1, "x_local must be a 1-D contiguous CUDA tensor")
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    st_obj = stream if stream is not None else torch.cuda.current_stream(x_local.device)
+    with torch.cuda.stream(st_obj):
+        if n_total is None:
+            t = torch.tensor([x_local.numel()], dtype=torch.int64, device=x_local.device)
+            n_total = int(_gather(t, group).sum().item())
+        if x_local.numel() != cyclic_local_len(n_total, chunk, world, rank):
+            raise SamError(-1, "x_local does not hold this rank's block-cyclic chunks of n_total elements")
+        if out is None:
+            out = torch.empty_like(x_local)
+        if lookahead is None:
+            lookahead = 0 if world == 1 else 1
+        gen = _cyclic_steps(x_local, out, order, tuple, inclusive, chunk, n_total, rank, world, lookahead, st_obj)
+        nccl = dist.get_backend(group) == "nccl"
+        pending = {}
+        try:
+            msg = next(gen)
+            while True:
+                if msg[0] == "send":
+                    r, pl = msg[1], msg[2]
+                    if world == 1:
+                        pending[r] = (None, pl)
+                    elif nccl:
+                        g = torch.empty(world * pl.numel(), dtype=torch.uint8, device=pl.device)
+                        pending[r] = (dist.all_gather_into_tensor(g, pl, group=group, async_op=True), g)
+                    else:
+                        pending[r] = (None, _gather(pl, group))
+                    msg = gen.send(None)
+                else:
+                    work, g = pending.pop(msg[1])
+                    if work is not None:
+                        work.wait()  # the compute stream waits for the collective (not the host)
+                    msg = gen.send(g)
+        except StopIteration:
+            pass
+    return out
+
+
+def scan_cyclic_virtual(x: torch.Tensor, nranks: int, chunk: int, order: int = 1, tuple: int = 1,
+                        inclusive: bool = True, lookahead: int = 1) -> torch.Tensor:
+    """The block-cyclic schedule of `nranks` virtual ranks on ONE GPU, in one process: each virtual
+    rank runs the same per-rank generator as scan_cyclic over its to_cyclic buffer; the exchange
+    is a concatenation once every rank has sent a round.  No kernel ever waits on another rank's
+    kernel (all on one stream, in an order where every round's payloads exist before its folds)."""
+    n = x.numel()
+    st_obj = torch.cuda.current_stream(x.device)
+    parts = [to_cyclic(x, chunk, nranks, g) for g in range(nranks)]
+    outs = [torch.empty_like(pt) for pt in parts]
+    gens = [_cyclic_steps(parts[g], outs[g], order, tuple, inclusive, chunk, n, g, nranks, lookahead, st_obj)
+            for g in range(nranks)]
+    sent: dict[int, list] = {}
+    ready: dict[int, torch.Tensor] = {}
+    msgs = [next(gen, None) for gen in gens]
+    while any(m is not None for m in msgs):
+        progress = False
+        for g in range(nranks):
+            while msgs[g] is not None:
+                m = msgs[g]
+                if m[0] == "send":
+                    row = sent.setdefault(m[1], [None] * nranks)
+                    row[g] = m[2].clone()
+                    if all(v is not None for v in row):
+                        ready[m[1]] = torch.cat(row)
+                    reply = None
+                elif m[1] in ready:
+                    reply = ready[m[1]]
+                else:
+                    break
+                try:
+                    msgs[g] = gens[g].send(reply)
+                except StopIteration:
+                    msgs[g] = None
+                progress = True
+        if not progress:
+            raise SamError(-5, "block-cyclic emulation made no progress")
+    return from_cyclic(outs, chunk, n)
 
 
 # ----------------------------------------------------------------------------- delta encoder
