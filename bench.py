@@ -265,6 +265,45 @@ def time_sharded(sam, synth, torch, dist, dt, n_local, k, s, rank, world, local,
     return res
 
 
+def time_cyclic(sam, synth, torch, dist, dt, n_local, k, s, rank, world, local, chunk=1 << 24, reps=3):
+    """One block-cyclic step (NEXT-1: per round a state pass over this rank's chunk, an all-gather of
+    the round's payloads, sam_cyclic_fold, the seeded scan of the chunk), max over ranks."""
+    from paper_conf_pldi_malekiyb16_b200.dist import cyclic_local_len, scan_cyclic, scan_cyclic_virtual
+
+    free, _ = torch.cuda.mem_get_info()
+    w = W_BYTES[dt]
+    if free < 2 * n_local * w + (3 << 30):
+        return {"skipped": f"needs {2 * n_local * w / 2**30:.0f} GiB free HBM per GPU"}
+    n_total = n_local * world
+    nl = cyclic_local_len(n_total, chunk, world, rank)
+    x = synth.make_torch(nl, dt, "uniform", seed=synth.SEED_BASE + 9, device=torch.device("cuda", local))
+    y = torch.empty_like(x)
+    st = torch.cuda.current_stream()
+    if world > 1:
+        fn = lambda: scan_cyclic(x, k, s, True, chunk=chunk, n_total=n_total, out=y)
+    else:
+        fn = lambda: scan_cyclic_virtual(x, 1, chunk, k, s, True, lookahead=0)
+    fn()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(reps):
+        fn()
+    e1.record(st)
+    torch.cuda.synchronize()
+    t = torch.tensor([e0.elapsed_time(e1) / reps], dtype=torch.float64, device=x.device)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t[0])
+    del x, y
+    torch.cuda.empty_cache()
+    return {"chunk": chunk, "step_ms": ms, "n_per_gpu": n_local, "n_total": n_total, "order": k, "tuple": s,
+            "dtype": DTYPE_NAME[dt], "gvalues_s": n_total / (ms * 1e-3) / 1e9,
+            "rounds": -(-(-(-n_total // chunk)) // world)}
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -320,6 +359,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-config sweep (C3/C4/C5) key")
+    ap.add_argument("--cyclic", action="store_true", help="also time the block-cyclic path at N=1 (always at N>1)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -553,6 +593,8 @@ def main():
         sharded = {}
         for tag, nl in (("c5_weak", 1 << 30), ("c5_strong", (1 << 33) // world)):
             sharded[tag] = time_sharded(sam, synth, torch, dist, "i64", nl, 4, 4, rank, world, local)
+        if world > 1 or args.cyclic:  # NEXT-1: the block-cyclic layout, C5 weak
+            sharded["cyclic_c5_weak"] = time_cyclic(sam, synth, torch, dist, "i64", 1 << 30, 4, 4, rank, world, local)
     alg_bytes = 2 * w * n_local
     achieved = alg_bytes / (kavg * 1e-3) / 1e9
     if rank == 0:

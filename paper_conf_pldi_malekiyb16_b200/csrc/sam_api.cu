@@ -72,8 +72,10 @@ struct Workspace {
     size_t carry_cap = 0;                 // bytes
     unsigned char* pend = nullptr;        // pending-state scratch (states > 16 B)
     size_t pend_cap = 0;
-    unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32][epoch u32][pad 16][seed 512 B]
+    unsigned char* ctr = nullptr;  // [tile_ctr u64][done u32][epoch u32][reset u32][state ticket u32][pad][seed 512 B]
+    unsigned char* part = nullptr; // state pass: per-CTA parts [grid][s][k] (fixed size, PART_BYTES)
 };
+constexpr size_t PART_BYTES = (size_t)2048 * 64 * 8;  // up to 2048 CTAs x 64 values x 8 B
 
 std::mutex g_mu;
 std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
@@ -289,6 +291,12 @@ void cyclic_fold_host_t(const unsigned char* P, size_t pb, int rank, int nranks,
     }
 }
 // block-cyclic fold on host buffers (sam_cyclic_fold_host)
+// SAM_STATE_VIA_SCAN=1 (read once): sam_shard_state runs the scan kernel in state-only mode (A/B)
+bool state_via_scan() {
+    static const bool v = getenv("SAM_STATE_VIA_SCAN") != nullptr && atoi(getenv("SAM_STATE_VIA_SCAN")) != 0;
+    return v;
+}
+
 int store_mode_for(const void* in, const void* out) {
     return ((((uintptr_t)in) ^ ((uintptr_t)out)) & 15) == 0 ? sam::STORE_BULK : sam::STORE_STRIPED;
 }
@@ -375,8 +383,30 @@ int sam_shard_state(sam_dtype dtype, int order, int tuple, const void* in_local,
     void* fs = (unsigned char*)payload_dev + 16;
     rc = payload_init(dtype, payload_dev, n_local, global_offset, order, tuple, nullptr, 1, fs, st);
     if (rc || n_local == 0) return rc;
-    return run_scan(dtype, order, tuple, 1, in_local, nullptr, n_local, global_offset, nullptr, fs,
-                    sam::STORE_NONE, st);
+    if (state_via_scan())  // A/B: the scan kernel in state-only mode (round 1-2 path)
+        return run_scan(dtype, order, tuple, 1, in_local, nullptr, n_local, global_offset, nullptr, fs,
+                        sam::STORE_NONE, st);
+    // the dedicated reduction kernel (sam_state.cuh): one read of the shard, no carry chain
+    Workspace* ws = nullptr;
+    int dev = 0;
+    rc = get_ws(st, 0, &ws, &dev);
+    if (rc) return rc;
+    if (!ws->part) {
+        cudaError_t e = cudaMalloc(&ws->part, PART_BYTES);
+        if (e != cudaSuccess) return fail(SAM_ERR_OOM, std::string("workspace: ") + cudaGetErrorString(e));
+    }
+    unsigned int* ticket = (unsigned int*)(ws->ctr + 20);
+    uint64_t l = 0;
+    cudaError_t e;
+    const int sms = num_sms_of(dev);
+    switch (add_dtype(dtype)) {
+        case SAM_I32: e = sam::launch_state<uint32_t>(in_local, n_local, global_offset, order, tuple, fs, ws->part, PART_BYTES, ticket, sms, st, &l); break;
+        case SAM_I64: e = sam::launch_state<uint64_t>(in_local, n_local, global_offset, order, tuple, fs, ws->part, PART_BYTES, ticket, sms, st, &l); break;
+        case SAM_F32: e = sam::launch_state<float>(in_local, n_local, global_offset, order, tuple, fs, ws->part, PART_BYTES, ticket, sms, st, &l); break;
+        default: e = sam::launch_state<double>(in_local, n_local, global_offset, order, tuple, fs, ws->part, PART_BYTES, ticket, sms, st, &l); break;
+    }
+    g_launches += l;
+    return e == cudaSuccess ? SAM_OK : cuda_fail(e, "state kernel launch");
 }
 
 int sam_shard_scan(sam_dtype dtype, int order, int tuple, int inclusive, const void* in_local, void* out_local,
@@ -745,6 +775,7 @@ int sam_release_workspaces(void) {
         Workspace* ws = kv.second;
         if (ws->carry) cudaFree(ws->carry);
         if (ws->ctr) cudaFree(ws->ctr);
+        if (ws->part) cudaFree(ws->part);
         delete ws;
     }
     g_ws.clear();

@@ -481,8 +481,12 @@ cudaError_t launch_payload_init(void* payload, uint64_t n, uint64_t g, int k, in
 
 }  // namespace sam
 
+#include "sam_state.cuh"
+
 #define SAM_INSTANTIATE(T)                                                                             \
     namespace sam {                                                                                    \
+    template cudaError_t launch_state<T>(const void*, uint64_t, uint64_t, int, int, void*, void*, size_t, \
+                                         unsigned int*, int, cudaStream_t, uint64_t*);                  \
     template cudaError_t launch_scan_tk<T, 1>(const LaunchArgs&, uint64_t*);                           \
     template cudaError_t launch_scan_tk<T, 2>(const LaunchArgs&, uint64_t*);                           \
     template cudaError_t launch_scan_tk<T, 3>(const LaunchArgs&, uint64_t*);                           \

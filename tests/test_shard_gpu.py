@@ -83,3 +83,40 @@ def test_seeded_scan_continues_a_stream():
     compare("i32", xn, out.cpu().numpy(), k, s, True)
     _, run = oracle.scan(xn, k, s, True)
     assert np.array_equal(st2.cpu().numpy().view(np.uint32).reshape(s, k), run.reshape(k, s).T)
+
+
+@pytest.mark.parametrize("name", ["i32", "i64", "f32", "f64"])
+@pytest.mark.parametrize("k,s", [(1, 1), (2, 1), (3, 3), (4, 4), (5, 2), (8, 8), (7, 5), (6, 6)])
+def test_state_kernel_payloads(name, k, s):
+    """The dedicated state-pass kernel (sam_state.cuh): the payload of sam_shard_state against the
+    oracle's running state, for n from 1 element to many tiles, global offsets with every lane
+    phase, and base pointers off the 16-B grid (the bulk copies' aligned superset)."""
+    import math
+
+    import paper_conf_pldi_malekiyb16_b200 as S
+
+    dc = {"i32": 0, "i64": 1, "f32": 2, "f64": 3}[name]
+    pb = S.sam_shard_payload_bytes(dc, k, s)
+    T = S.tile_items(name) * 256 if hasattr(S, "tile_items") else 3328
+    for n, g, off in [(1, 0, 0), (5, 3, 1), (T - 1, 7, 0), (T + 1, 1, 3), (3 * T + 17, 0, 2), (100_003, 12345, 1),
+                      (1_000_003, 5, 0)]:
+        kind = "uniform" if name.startswith("i") else "small"
+        xn = synth.make(n + 4, name, kind, seed=n + k * 8 + s)
+        x = torch.from_numpy(xn).cuda()
+        w = x.element_size()
+        pay = torch.zeros(pb, dtype=torch.uint8, device="cuda")
+        S.sam_shard_state(dc, k, s, ctypes.c_void_p(x.data_ptr() + off * w), n, g, ctypes.c_void_p(pay.data_ptr()))
+        torch.cuda.synchronize()
+        ph = pay.cpu().numpy()
+        assert int(ph[:16].view(np.uint64)[0]) == n and int(ph[:16].view(np.uint64)[1]) == g
+        seg = xn[off:off + n]
+        _, run = oracle.scan(seg, k, s, True, phase=g % s)
+        ref = run.reshape(k, s).T
+        if name.startswith("i"):
+            got = ph[16:16 + k * s * w].view(ref.dtype).reshape(s, k)
+            assert np.array_equal(got, ref), f"n={n} g={g} off={off}"
+        else:
+            got = ph[16:16 + k * s * w].view(np.float32 if name == "f32" else np.float64).reshape(s, k).astype(np.float64)
+            A = oracle.scan(np.abs(seg), k, s, True, phase=g % s)[1].reshape(k, s).T.astype(np.float64)
+            tol = (1e-5 if name == "f32" else 1e-12) * math.sqrt(max(1, n) * k) * A
+            assert (np.abs(got - ref.astype(np.float64)) <= tol).all(), f"n={n} g={g} off={off}"
