@@ -17,3 +17,10 @@ timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_d
     --clock-control none --csv --log-file gpurun_out/ncu_sweep.csv python tools/ncu_sweep.py > gpurun_out/ncu_sweep.log 2>&1
 timeout 600 python tools/ablation.py gpurun_out/ablation.json > gpurun_out/ablation.txt 2>&1
 ls -la gpurun_out
+# the dedicated state-pass kernel on north_star's multi-GPU config (C5 shard, 2^30 int64 k=4 s=4)
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:sam_state_kernel -s 2 -c 1 \
+   -o gpurun_out/full_state_i64_k4_s4 python tools/prof_state.py i64 30 4 4 > gpurun_out/full_state.log 2>&1
+python tools/ncu_summary.py gpurun_out/full_state_i64_k4_s4.ncu-rep > gpurun_out/full_state_i64_k4_s4.txt 2>&1
+rm -f gpurun_out/full_state_i64_k4_s4.ncu-rep
+timeout 600 python tools/state_bench.py > gpurun_out/state_bench.txt 2>&1
+ls -la gpurun_out
