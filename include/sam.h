@@ -143,7 +143,8 @@ int sam_scan_host(sam_dtype dtype, int order, int tuple, int inclusive, const vo
 
 /* ---------------------------------------------------------------------------------------
  * Sharded (multi-GPU) scan: contiguous shards in rank order.
- *   1. sam_shard_state: read-only pass over the local shard -> payload (device memory,
+ *   1. sam_shard_state: read-only pass over the local shard (a dedicated reduction kernel, no
+ *      carry chain: partial lane states combine with the carry operator in any grouping) -> payload (device memory,
  *      sam_shard_payload_bytes bytes): [u64 n_local][u64 global_offset][order*tuple values,
  *      [lane][order]], padded to a multiple of 16 B] = the zero-seeded state of each global lane at its last element of the
  *      shard.
@@ -178,8 +179,9 @@ int sam_fold_payloads_host(sam_dtype dtype, int order, int tuple, const void* al
  * (one per rank).  Per round each rank (1) runs sam_shard_state on its chunk (global offset
  * c*C) while the chunk stays in L2, (2) all ranks exchange the p payloads of the round, (3)
  * sam_cyclic_fold gives the carry into its chunk, (4) sam_scan_seeded scans the chunk (its re-read
- * an L2 hit), so each element costs one HBM read and one write on every GPU -- contiguous shards
- * cost 1.5x that (state pass over the whole shard, then the scan).
+ * an L2 hit when the chunk fits there), so each element costs one HBM read and one write on every
+ * GPU -- contiguous shards cost 1.5x that (state pass over the whole shard, then the scan).  Each
+ * round is three kernel launches, so chunks must be large enough to amortise them.
  *
  * sam_cyclic_fold: `round_payloads` (device, nranks * sam_shard_payload_bytes, rank order) = the
  * payloads of one round; `base_in` (device, [tuple][order], or NULL = zero state) = the state of

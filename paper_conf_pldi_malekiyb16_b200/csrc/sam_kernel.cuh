@@ -26,7 +26,7 @@
 //                   outputs (the binomial fix-up C(r+t-j, t-j)); exclusive = inclusive shifted by
 //                   k lane positions (R1), the first k from finite differences.
 //                   A loaded tile's local scan always goes first (its aggregate gates other
-//                   CTAs' look-backs); up to LAG tiles may await their carries.
+//                   CTAs' carry folds); up to LAG tiles may await their carries.
 //   aggregator warp a3/a4: combines the warp states of a tile and publishes its per-lane k-vector
 //                   aggregate (one value per order; all s lanes).
 //   carry warps     a5: SAM's carry scheme on a static schedule: the carry into
@@ -52,7 +52,7 @@ namespace sam {
 
 template <typename T> struct Cfg;
 // ITEMS odd (bank-conflict-free strided smem reads); NB1 / NB2 smem buffers for local scans / carry
-// application + store; LAG = max tiles between local scan and carry application (the look-back's
+// application + store; LAG = max tiles between local scan and carry application (the carry fold's
 // latency budget, states in registers); PF = max claimed-but-unscanned tiles per CTA.
 template <> struct Cfg<uint32_t> { static constexpr int ITEMS = 27; };
 template <> struct Cfg<float>    { static constexpr int ITEMS = 27; };
@@ -114,7 +114,7 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_EARLY_RELOAD
 #define SAM_EARLY_RELOAD 0
 #endif
-// back-off (ns) of the look-back re-polls, of idle compute warps and of the idle producer
+// back-off (ns) of the carry-fold re-polls, of idle compute warps and of the idle producer
 #ifndef SAM_POLL_NS
 #define SAM_POLL_NS 0
 #endif
@@ -148,6 +148,10 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_MMAX_BIG
 #define SAM_MMAX_BIG 2
 #endif
+// states > 16 B too: separate local-scan / carry-application warp groups (pending states in L2)
+#ifndef SAM_SPLIT_BIG
+#define SAM_SPLIT_BIG 0
+#endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
 #endif
@@ -180,18 +184,18 @@ template <typename T, int K> struct Lag {
     static constexpr bool GPEND = SAM_GPEND && SB > 16;
     static constexpr bool SMEM = !GPEND && (SB <= 16 || BIG32 || BIG64);  // pending local states in shared memory
     static constexpr int LAG = GPEND ? SAM_LAGG : (SB <= 4 ? SAM_LAG_SMALL : (SB <= 8 ? SAM_LAG8 : (SB <= 16 ? SAM_LAG16 : (BIG32 ? SAM_LAG32 : SAM_LAG64))));
-    // max tiles per super-tile (look-back unit); measured: 3 for 4-byte, 2 for 8-byte elements
+    // max tiles per super-tile (carry unit); measured: 3 for 4-byte, 2 for 8-byte elements
     static constexpr int MMAX = (SB <= 8 && sizeof(T) == 4) ? 3 : (SB <= 8 ? 2 : SAM_MMAX_BIG);
     static constexpr int NB1 = 3;                    // local-scan (HBM) buffers
     static constexpr int NB2 = SB <= 8 ? 4 : 2;      // carry-application (L2 reload) buffers
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = SB <= 16 && K >= SAM_SPLIT_MIN_K;
+    static constexpr bool SPLIT = (SB <= 16 || SAM_SPLIT_BIG) && K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int NCARRY = 4;                          // carry (look-back) warps
+constexpr int NCARRY = 4;                          // carry warps (the fold of each super-tile's carry)
 constexpr int NCARRY_P1 = NCARRY + 1;
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
@@ -206,7 +210,7 @@ enum StoreMode { STORE_BULK = 0, STORE_STRIPED = 1, STORE_NONE = 2 };
 
 // 64-bit tagged words per value: 1 for 32-bit types ([tag|value]), 2 for 64-bit ([tag|lo],[tag|hi])
 template <typename T> struct TagW { static constexpr int W = sizeof(T) == 4 ? 1 : 2; };
-// look-back window rows per round trip (carry-warp register budget: V*K*2W <= 16 words per lane)
+// carry-fold window rows per round trip (carry-warp register budget: V*K*2W <= 16 words per lane)
 template <typename T, int K> struct LB {
     static constexpr int W1 = TagW<T>::W;
     static constexpr int V0 = 16 / (K * W1);
@@ -228,7 +232,7 @@ struct Params {
     uint64_t h;          // virtual index of in[0] (= lane phase, 0 <= h < s)
     uint64_t num_tiles;  // ceil((h + n) / T)
     uint64_t num_super;  // ceil(num_tiles / M)
-    int M;               // tiles per super-tile (look-back unit), 1..MMAX
+    int M;               // tiles per super-tile (carry unit), 1..MMAX
     uint32_t delta;      // byte offset of virtual element 0 inside its 16-B chunk
     int s, G, logG, sp, c, logc, Pw, W, Wn;
     int U, T_, Uw;
@@ -476,7 +480,7 @@ struct SmemL {
     static constexpr int NQ = (LAG + 1 > NB1 ? LAG + 1 : NB1) + 1;  // per-iteration state ring
     static constexpr int ELAG = Lag<T, K>::SMEM ? LAG : 0;          // smem-resident pending states
     static constexpr int TMAX = TILE_THREADS * ITEMS;
-    static constexpr int NBL = 32;                // look-back binomial rows
+    static constexpr int NBL = 32;                // carry-fold binomial rows
     static constexpr int BUFB = ((TMAX * (int)sizeof(T) + 32) + 127) / 128 * 128;
     static constexpr int WQ = (VEC ? 8 : 64) * K; // per-iteration warp states [pairs][K] (VEC: s = 1, 8 warps)
     static constexpr int LA = 8 * K;              // per-iteration tile aggregate [8][K]
@@ -779,7 +783,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // Per tile: combine the warp states (E = warp-exclusive prefixes, tile aggregate A_j); per
         // super-tile: the running prefix P_j = A_0 (+) ... (+) A_{j-1} (kept in registers by the
         // lane that owns lane m's aggregate), and after the last sub-tile the super-tile aggregate,
-        // published for the other CTAs' look-backs (a4).
+        // published for the other CTAs' carry folds (a4).
         const int npair = s * c;
         T Pref[2][K];
         T gneg[K];  // global frame (integers): b(-(S+1) US) of this CTA's current super-tile
@@ -1904,8 +1908,14 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     while (flag_ld_acq(p2_cnt) < (i - lag + 1) * NW) __nanosleep(32);
                     T e[K];
                     local_scan(i, b1, e);
+                    if constexpr (EGMEM) {
+                        T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % LAG)) * K * TILE_THREADS + gtid;
 #pragma unroll
-                    for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                        for (int t = 0; t < K; ++t) pe[t * TILE_THREADS] = e[t];
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t] = e[t];
+                    }
                 }
             } else {
                 for (int i = 0;; ++i) {
@@ -1913,8 +1923,14 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                     if (!wait_or_end(&bar_full2[b2], (uint32_t)((i / NB2) & 1), i)) break;
                     if (SAM_EARLY_RELOAD) mbar_wait(&bar_carry[i % NQ], (uint32_t)((i / NQ) & 1));
                     T e[K];
+                    if constexpr (EGMEM) {
+                        const T* pe = p.pend + ((size_t)blockIdx.x * LAG + (i % LAG)) * K * TILE_THREADS + gtid;
 #pragma unroll
-                    for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
+                        for (int t = 0; t < K; ++t) e[t] = pe[t * TILE_THREADS];
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < K; ++t) e[t] = eq_s[((i % LAG) * TILE_THREADS + gtid) * K + t];
+                    }
                     carry_apply(i, tile_of[i % NQ], e);
                     __syncwarp();
                     if (lane == 0) {
@@ -1925,7 +1941,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
             }
         } else {
             // One group.  A loaded tile's local scan (P1) always goes first, so its aggregate is
-            // published as early as possible (predecessor aggregates gate every look-back); a
+            // published as early as possible (predecessor aggregates gate every carry fold); a
             // tile's carry application (P2) runs once the producer has re-fetched it.  Up to LAG
             // tiles sit between P1 and P2, their local states in registers (static ring eq).
             T eq[(ESMEM || EGMEM) ? 1 : LAG][K];  // register ring only when the states are in neither smem nor L2
