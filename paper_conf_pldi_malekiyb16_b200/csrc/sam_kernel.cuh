@@ -148,9 +148,14 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
 #ifndef SAM_MMAX_BIG
 #define SAM_MMAX_BIG 2
 #endif
-// states > 16 B too: separate local-scan / carry-application warp groups (pending states in L2)
+// 8-byte states of up to SAM_SPLIT_MAXB bytes (int64 order 3) also get the two warp groups, their
+// pending states in L2: 22 warps cap registers at 80, which order 3 fits without spills (measured
+// +17% int64 k=3, +38% int64 k=3 s=3; orders >= 4 spill and lose, profiles/r2b_ab_splitbig.txt)
 #ifndef SAM_SPLIT_BIG
-#define SAM_SPLIT_BIG 0
+#define SAM_SPLIT_BIG 1
+#endif
+#ifndef SAM_SPLIT_MAXB
+#define SAM_SPLIT_MAXB 24
 #endif
 #ifndef SAM_SPLIT_MIN_K
 #define SAM_SPLIT_MIN_K 2
@@ -191,11 +196,15 @@ template <typename T, int K> struct Lag {
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = (SB <= 16 || SAM_SPLIT_BIG) && K >= SAM_SPLIT_MIN_K;
+    static constexpr bool SPLIT = (SB <= 16 || (SAM_SPLIT_BIG && sizeof(T) == 8 && SB <= SAM_SPLIT_MAXB)) &&
+                                  K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
-constexpr int NCARRY = 4;                          // carry warps (the fold of each super-tile's carry)
+#ifndef SAM_NCARRY
+#define SAM_NCARRY 4
+#endif
+constexpr int NCARRY = SAM_NCARRY;                 // carry warps (the fold of each super-tile's carry)
 constexpr int NCARRY_P1 = NCARRY + 1;
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
@@ -769,7 +778,7 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
                         SAM_STRESS(0, t);
                         load_tile(t, smem + S::OFF_BUF1 + (j1 % NB1) * S::BUFB, &bar_full1[j1 % NB1], pol_keep);
                         ++j1;
-                        flag_st_rel(claimed, j1);  // tile_of / sup_of / sub_of of iteration j1-1 are set
+                        if (p.dyn) flag_st_rel(claimed, j1);  // tile_of / sup_of / sub_of of iteration j1-1 are set
                     }
                     continue;
                 }

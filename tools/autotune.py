@@ -11,14 +11,15 @@ import paper_conf_pldi_malekiyb16_b200 as S  # noqa: E402
 import synth  # noqa: E402
 
 quick = "--quick" in sys.argv
-OUT = os.path.join(os.path.dirname(S.LIB_PATH), "sam_tune.txt")
+OUT = next((a.split("=", 1)[1] for a in sys.argv if a.startswith("--out=")),
+           os.path.join(os.path.dirname(S.LIB_PATH), "sam_tune.txt"))
 TY = {"i32": "u32", "i64": "u64", "f32": "f32", "f64": "f64"}
 classes = [(dt, k, s) for dt in ("i32", "i64") for k in (1, 2, 3, 4, 5, 6, 7, 8) for s in (1, 2, 3, 4, 5, 6, 7, 8)
            if k * s <= 16 or (k, s) in ((4, 4), (2, 8), (8, 2), (8, 8))]
 classes += [(dt, 1, s) for dt in ("f32", "f64") for s in (1, 2, 4, 8)]
 if quick:
     classes = [c for c in classes if c[1] in (1, 2, 4, 8) and c[2] in (1, 2, 4, 8)]
-ranges = [(20, 24, 22), (25, 33, 28)]  # (log2 lo, log2 hi, measured at)
+ranges = [(20, 24, 22), (25, 28, 28), (29, 33, 30)]  # (log2 lo, log2 hi, measured at)
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 lines = []
 bufs = {}
