@@ -196,8 +196,6 @@ template <typename T, int K> struct Lag {
     static constexpr int PF = NB1;                   // max claimed-but-unscanned tiles
     // orders 2..4 with smem-resident pending states: separate warp groups for local scans (P1) and
     // carry applications (P2) (measured faster there; order 1 keeps one group)
-    static constexpr bool SPLIT = (SB <= 16 || (SAM_SPLIT_BIG && sizeof(T) == 8 && SB <= SAM_SPLIT_MAXB)) &&
-                                  K >= SAM_SPLIT_MIN_K;
 };
 
 constexpr int MAX_CWARPS = 8;                      // compute warps
@@ -208,10 +206,23 @@ constexpr int NCARRY = SAM_NCARRY;                 // carry warps (the fold of e
 constexpr int NCARRY_P1 = NCARRY + 1;
 constexpr int SERVICE_WARPS = 2 + NCARRY;          // producer + aggregator + carry warps
 constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
-// threads of a CTA: one compute group (or two: local scans + carry applications) + service warps
-template <typename T, int K> struct Threads {
-    static constexpr int GROUPS = Lag<T, K>::SPLIT ? 2 : 1;
-    static constexpr int VALUE = (GROUPS * MAX_CWARPS + SERVICE_WARPS) * 32;
+// Warp roles of one instantiation.  NC carry warps: 2 for the 128-bit tuple-1 kernels of orders >= 2
+// (their folds are small -- s*k <= 8 values -- and the two warps' registers go to the compute warps;
+// measured +5..+19% for int32 k=4,8 and int64 k=2,4,5,8; int32 k=2 and int64 k=3 keep four:
+// profiles/r2b_ab_ncarry.txt), else 4.  SPLIT: separate warp
+// groups for local scans and carry applications -- states <= 16 B, and 8-byte states up to 24 B (32 B
+// with two carry warps), the register cap of the larger CTA still holding them without spills.
+#ifndef SAM_NC_VEC2
+#define SAM_NC_VEC2 1
+#endif
+template <typename T, int K, bool VEC> struct Threads {
+    static constexpr int SB = K * (int)sizeof(T);
+    static constexpr int NC =
+        (SAM_NC_VEC2 && VEC && K >= 2 && !(sizeof(T) == 4 && K == 2) && !(sizeof(T) == 8 && K == 3)) ? 2 : NCARRY;
+    static constexpr bool SPLIT =
+        (SB <= 16 || (SAM_SPLIT_BIG && sizeof(T) == 8 && SB <= (NC == 2 ? 32 : SAM_SPLIT_MAXB))) && K >= SAM_SPLIT_MIN_K;
+    static constexpr int GROUPS = SPLIT ? 2 : 1;
+    static constexpr int VALUE = (GROUPS * MAX_CWARPS + 2 + NC) * 32;
 };
 constexpr int TILE_THREADS = MAX_CWARPS * 32;
 
@@ -542,7 +553,7 @@ struct Smem : SmemPick<T, K, VEC>::type {};
 // the kernel
 // ------------------------------------------------------------------------------------------
 template <typename T, int K, bool VEC>
-__global__ void __launch_bounds__(Threads<T, K>::VALUE, 1)
+__global__ void __launch_bounds__(Threads<T, K, VEC>::VALUE, 1)
 sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     using S = Smem<T, K, VEC>;
     using CT = typename Coef<T>::type;
@@ -593,7 +604,8 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
     const int s = p.s, c = p.c;
-    constexpr bool SPLIT = Lag<T, K>::SPLIT;
+    constexpr bool SPLIT = Threads<T, K, VEC>::SPLIT;
+    constexpr int NC = Threads<T, K, VEC>::NC;  // carry warps (ring depths stay NCARRY)
     const int NW = p.W;          // compute warps per group
     const int NCT = NW * 32;     // compute threads per group
     const int NCW = SPLIT ? 2 * NW : NW;  // compute warps (both groups); service warps follow
@@ -993,10 +1005,10 @@ sam_scan_kernel(const __grid_constant__ Params<T, K> p) {
         // Teams: the carry warps form NT teams of TW warps; team t takes this CTA's super-tiles t, t+NT,
         // ... (folds of successive super-tiles overlap; only the short chain step is ordered, through
         // the hand-off entries).  coop = 0 is NT = 4 teams of one warp.
-        const int NT = coop ? (p.teams == 2 ? 2 : 1) : NCARRY;  // 1, 2 or 4 (no divisions below)
+        const int NT = coop ? (p.teams == 2 && NC >= 2 ? 2 : 1) : NC;  // 1, 2 or NC teams
         const int lgNT = NT == 1 ? 0 : (NT == 2 ? 1 : 2);
-        const int TW = NCARRY >> lgNT;
-        const int team = cw >> (2 - lgNT), tw = cw - team * TW;
+        const int TW = NC >> lgNT;
+        const int team = cw / TW, tw = cw - team * TW;
         const bool lead = tw == 0;  // finishes the super-tile (hand-off, sub-tile states)
         const int WV = p.Wn * p.Vr;          // super-tiles per window
         CT* const part_s = (CT*)(smem + S::OFF_PART);  // [2][NCARRY][MAXS][K] coop partial folds

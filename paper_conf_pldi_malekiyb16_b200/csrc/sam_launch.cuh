@@ -285,7 +285,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
                                                  cudaFuncAttributeMaxDynamicSharedMemorySize, S::BYTES);
             if (e != cudaSuccess) return e;
             int nb = 0;
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K, VEC>, Threads<T, K>::VALUE, S::BYTES);
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sam_scan_kernel<T, K, VEC>, Threads<T, K, VEC>::VALUE, S::BYTES);
             if (e != cudaSuccess) return e;
             info.max_blocks_per_sm[dev] = nb > 0 ? nb : 1;
             info.ready[dev] = true;
@@ -420,7 +420,7 @@ cudaError_t launch_scan_impl(const LaunchArgs& a, uint64_t* launches) {
         cudaLaunchConfig_t cfg;
         memset(&cfg, 0, sizeof(cfg));
         cfg.gridDim = dim3((unsigned)P);
-        cfg.blockDim = dim3((Threads<T, K>::GROUPS * geo.W + SERVICE_WARPS) * 32);
+        cfg.blockDim = dim3((Threads<T, K, VEC>::GROUPS * geo.W + 2 + Threads<T, K, VEC>::NC) * 32);
         cfg.dynamicSmemBytes = S::BYTES;
         cfg.stream = a.stream;
         cudaLaunchAttribute attr[1];
