@@ -2,7 +2,9 @@
     python tools/sweep.py [reps]"""
 import sys, os, statistics
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import time
 import torch, synth
+SOAK = float(os.environ.get("SOAK", "0"))
 import paper_conf_pldi_malekiyb16_b200 as S
 reps = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 cfgs = [("i32", 30, 1, 1), ("i32", 28, 1, 1), ("i64", 28, 1, 1), ("i32", 28, 2, 1), ("i64", 28, 2, 1),
@@ -24,6 +26,11 @@ for r in range(reps):
         dt, logn, k, s = c
         x, y = data[c]
         for _ in range(2): S.scan(x, k, s, True, out=y)
+        if SOAK > 0:  # sustained: run the config alone for SOAK seconds first (power-cap clocks)
+            t0 = time.time()
+            while time.time() - t0 < SOAK:
+                for _ in range(5): S.scan(x, k, s, True, out=y)
+                torch.cuda.synchronize()
         torch.cuda.synchronize(); e0.record()
         it = 10
         for _ in range(it): S.scan(x, k, s, True, out=y)
