@@ -214,6 +214,9 @@ constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
 // with two carry warps), the register cap of the larger CTA still holding them without spills.
 // 4-byte states of 20..32 B (int32 orders 5-8) with two carry warps: split too (96 registers, no spills;
 // sustained +1/+7/+20/+14% at orders 5/6/7/8, profiles/r2b_ab_split4b.txt)
+#ifndef SAM_SPLIT_NV
+#define SAM_SPLIT_NV 1
+#endif
 #ifndef SAM_SPLIT_4B
 #define SAM_SPLIT_4B 1
 #endif
@@ -226,7 +229,7 @@ template <typename T, int K, bool VEC> struct Threads {
         (SAM_NC_VEC2 && VEC && K >= 2 && !(sizeof(T) == 4 && K == 2) && !(sizeof(T) == 8 && K == 3)) ? 2 : NCARRY;
     static constexpr bool SPLIT =
         (SB <= 16 || (SAM_SPLIT_BIG && (sizeof(T) == 8 || (SAM_SPLIT_4B && NC == 2)) && SB <= (NC == 2 ? 32 : SAM_SPLIT_MAXB))) &&
-        K >= SAM_SPLIT_MIN_K;
+        K >= SAM_SPLIT_MIN_K && (VEC || SAM_SPLIT_NV);
     static constexpr int GROUPS = SPLIT ? 2 : 1;
     static constexpr int VALUE = (GROUPS * MAX_CWARPS + 2 + NC) * 32;
 };
