@@ -120,3 +120,13 @@ def test_C5_2p33_int64_order4_tuple4_single_gpu():
         ref, run = oracle.scan(xc, k, s, True, phase=off % s, run=run)
         got = y[off:off + chunk].cpu().numpy().view(ref.dtype)
         assert np.array_equal(got, ref), f"mismatch in chunk at {off}"
+    # the state-pass reduction kernel (sam_shard_state) over the same 2^33 elements: the zero-seeded
+    # state of every lane at its last element = the chunked oracle's final running sums
+    import ctypes
+
+    pay = torch.zeros(S.sam_shard_payload_bytes(S.SAM_I64, k, s), dtype=torch.uint8, device="cuda")
+    S.sam_shard_state(S.SAM_I64, k, s, ctypes.c_void_p(x.data_ptr()), n, 0, ctypes.c_void_p(pay.data_ptr()))
+    torch.cuda.synchronize()
+    st = pay.cpu().numpy()[16:16 + 8 * k * s].view(np.uint64).reshape(s, k)
+    assert np.array_equal(st, np.asarray(run).reshape(k, s).T.view(np.uint64)), "state pass at 2^33"
+
