@@ -222,9 +222,13 @@ constexpr int MAX_THREADS = (MAX_CWARPS + SERVICE_WARPS) * 32;
 #endif
 // 8-byte order-1 tuple kernels: their fold is a plain sum of s values, two carry warps suffice
 // (measured int64 k=1 s=2..7 +1..+8%, s=8 -5%, fp64 s=2/5/8 +2/+10/+2%; 4-byte tuples lose 3-7%:
-// profiles/r2b_ab_nc2_tuples.txt, r2b_ab_nc2_t8k1.txt)
+// profiles/r2b_ab_nc2_tuples.txt, r2b_ab_nc2_t8k1.txt); the 128-bit tuple-1 kernels too (int64 +3%, fp64 +5%,
+// profiles/r2b_ab_nc2_t8k1v.txt)
 #ifndef SAM_NC_T8K1
 #define SAM_NC_T8K1 1
+#endif
+#ifndef SAM_NC_T8K1V
+#define SAM_NC_T8K1V 1
 #endif
 #ifndef SAM_NC_VEC2
 #define SAM_NC_VEC2 1
@@ -233,7 +237,7 @@ template <typename T, int K, bool VEC> struct Threads {
     static constexpr int SB = K * (int)sizeof(T);
     static constexpr int NC =
         ((SAM_NC_VEC2 && VEC && K >= 2 && !(sizeof(T) == 4 && K == 2) && !(sizeof(T) == 8 && K == 3)) ||
-         (SAM_NC_T8K1 && !VEC && sizeof(T) == 8 && K == 1)) ? 2 : NCARRY;
+         (SAM_NC_T8K1 && (!VEC || SAM_NC_T8K1V) && sizeof(T) == 8 && K == 1)) ? 2 : NCARRY;
     static constexpr bool SPLIT =
         (SB <= 16 || (SAM_SPLIT_BIG && (sizeof(T) == 8 || (SAM_SPLIT_4B && NC == 2)) && SB <= (NC == 2 ? 32 : SAM_SPLIT_MAXB))) &&
         K >= SAM_SPLIT_MIN_K && (VEC || SAM_SPLIT_NV);
