@@ -100,11 +100,14 @@ __device__ __forceinline__ void sts_vec(T* p, const T (&d)[N]) {
         reinterpret_cast<uint4*>(p)[q] = v;
     }
 }
-// Pipeline shape by per-thread state size K * sizeof(T):
-//   <= 8 B : 3 local-scan buffers, 3 carry buffers, pending states in smem (LAG = 12), super-tiles of 4
-//   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8), super-tiles of 2
-//   larger : 3 + 2 buffers, pending states in registers (LAG = 4), super-tiles of 2
-// (SAM_LAG_SMALL / SAM_SPLIT_MIN_K: compile-time overrides for experiments, tools/build_variant.py)
+// Pipeline shape by per-thread state size K * sizeof(T) (struct Lag below):
+//   <= 8 B : 3 local-scan buffers, 4 carry buffers, pending states in smem (LAG = 12)
+//   <= 16 B: 3 + 2 buffers, pending states in smem (LAG = 8)
+//   larger : 3 + 2 buffers, pending states in an L2-resident global scratch (LAG = 8)
+// super-tile sizes (tiles per carry unit) come from the launch (MMAX, the autotune table); warp roles
+// (carry warps, split compute groups) from struct Threads.  The SAM_* macros are compile-time overrides
+// for experiments (tools/build_variant.py).  (Pending states <= 16 B in smem since round 1, larger ones in
+// global scratch since round 2.)
 #ifndef SAM_LAG_SMALL
 #define SAM_LAG_SMALL 12
 #endif
